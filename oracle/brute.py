@@ -1,0 +1,127 @@
+"""O2: brute force over all G^N GPU labelings (TEST INFRASTRUCTURE ONLY, N <= 6).
+
+Independent of enum.c: the space is built by canonicalising every labeling
+of the N workflows onto G GPUs (GPUs are interchangeable -> relabel blocks by
+first occurrence, "groups ... on available GPUs"), the index
+order is obtained by SORTING the distinct (RGS, level digits) tuples
+(reading R4: RGS lexicographic, then digits most-significant first), and
+each configuration is scored by a separate pure-Python fp64 transcription
+of the canonical score (PAPER.md L87, L91, L96,
+L116).  Python floats are IEEE binary64 with one rounding per operation.
+"""
+from __future__ import annotations
+
+import itertools
+
+PER_CLIENT = 0
+
+
+def space(n, g, c, L, scope):
+    """Sorted list of (rgs, digits) for the whole space."""
+    rgss = set()
+    for lab in itertools.product(range(g), repeat=n):
+        m = {}
+        rgs = tuple(m.setdefault(x, len(m)) for x in lab)
+        k = len(m)
+        sizes = [rgs.count(b) for b in range(k)]
+        if max(sizes) <= c:
+            rgss.add(rgs)
+    out = []
+    for rgs in sorted(rgss):
+        k = max(rgs) + 1
+        nd = n if scope == PER_CLIENT else k
+        for dig in itertools.product(range(L), repeat=nd):
+            out.append((rgs, dig))
+    return out
+
+
+def t_seq(t100, g):
+    fin = [0.0] * g
+    for ti in t100:
+        j = min(range(g), key=lambda x: (fin[x], x))
+        fin[j] = fin[j] + ti
+    return max(fin)
+
+
+def e_seq(p100, t100):
+    e = 0.0
+    for pi, ti in zip(p100, t100):
+        e = e + pi * ti
+    return e
+
+
+def score(prof, n, rgs, lv_prof):
+    """lv_prof[i]: profile level index of workflow i. -> (feasible, T, E)."""
+    t = prof.solo_time_s.astype(float)
+    p = prof.solo_power_w.astype(float)
+    u = prof.sm_util.astype(float)
+    bw = prof.bw_util.astype(float)
+    d = prof.corun_slowdown.astype(float)
+    ps = float(prof.static_power_w)
+    k = max(rgs) + 1
+    groups = [[i for i in range(n) if rgs[i] == b] for b in range(k)]
+    for grp in groups:
+        if sum(int(prof.max_mem_mib[i]) for i in grp) > int(prof.mem_capacity_mib):
+            return False, None, None
+    T = 0.0
+    E = 0.0
+    for grp in groups:
+        U = 0.0
+        B = 0.0
+        for i in grp:
+            U = U + u[i, lv_prof[i]]
+            B = B + bw[i, lv_prof[i]]
+        cg = max(max(1.0, U), B)
+        Tg = 0.0
+        for i in grp:
+            s = 1.0
+            for j in grp:
+                if j != i:
+                    s = s + d[i, lv_prof[i], j, lv_prof[j]]
+            tau = (t[i, lv_prof[i]] * s) * cg
+            Tg = max(Tg, tau)
+        D = 0.0
+        for i in grp:
+            D = D + (p[i, lv_prof[i]] - ps) * t[i, lv_prof[i]]
+        T = max(T, Tg)
+        E = E + (ps * Tg + D)
+    return True, T, E
+
+
+def search(prof, q):
+    pct = [int(x) for x in prof.level_pct]
+    lev = [pct.index(v) for v in q.levels]
+    l100 = pct.index(100)
+    t100 = [float(prof.solo_time_s[i, l100]) for i in range(q.n)]
+    p100 = [float(prof.solo_power_w[i, l100]) for i in range(q.n)]
+    ts = t_seq(t100, q.g)
+    es = e_seq(p100, t100)
+    sp = space(q.n, q.g, min(q.c, q.n), len(q.levels), q.scope)
+    best = [None] * len(q.weights)
+    feas = []
+    for idx, (rgs, dig) in enumerate(sp):
+        lvp = [lev[dig[i]] if q.scope == PER_CLIENT else lev[dig[rgs[i]]] for i in range(q.n)]
+        ok, T, E = score(prof, q.n, rgs, lvp)
+        if not ok:
+            continue
+        feas.append((idx, T, E))
+        X = ts / T
+        Y = es / E
+        for w, (a, b) in enumerate(q.weights):
+            F = 1.0
+            for _ in range(a):
+                F = F * X
+            for _ in range(b):
+                F = F * Y
+            if best[w] is None or F > best[w][1]:
+                best[w] = (idx, F, T, E)
+    # Pareto by O(n^2) definition: not dominated by any feasible config;
+    # one (lowest) index per distinct (T, E).
+    pts = {}
+    for idx, T, E in feas:
+        dom = any((T2 <= T and E2 <= E) and (T2 < T or E2 < E) for _, T2, E2 in feas)
+        if not dom and (T, E) not in pts:
+            pts[(T, E)] = idx
+    pareto = sorted([(i, T, E) for (T, E), i in pts.items()], key=lambda x: (x[1], x[2], x[0]))
+    return dict(best=best, pareto=pareto, nconfigs=len(sp), nfeasible=len(feas),
+                tseq=ts, eseq=es, space=sp)
