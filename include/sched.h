@@ -1,0 +1,194 @@
+/*
+ * sched.h -- C ABI of the B200 exhaustive co-scheduling configuration search.
+ *
+ * The hot path of the granularity- and interference-aware MPS scheduler of
+ * Weaver et al., "Granularity- and Interference-Aware GPU Sharing with MPS"
+ * (SC'24 workshops).  PAPER.md below is /root/reference/PAPER.md; R<n> are
+ * the readings of the paper listed in DESIGN.md ("Readings of the paper").
+ *
+ * Problem statement (Sec. IV-B): "we select groups of queued
+ * workflows to co-schedule on available GPUs based on (1) predicted
+ * interference and (2) evaluation metric priority (i.e., optimize throughput
+ * or energy)".  The library scores EVERY configuration -- a set partition of
+ * the queued workflows 0..n-1 into k <= g MPS client groups (one group per
+ * GPU, <= max_clients members) times an MPS active-thread
+ * level per client (PER_CLIENT) or per GPU (PER_GPU) (granularity, PAPER.md
+ * L75) -- for throughput X = T_seq/T and energy efficiency Y = E_seq/E
+ * relative to sequential scheduling, and returns the best
+ * configuration for each product metric X^a * Y^b and
+ * the exact throughput/energy Pareto set.  The score is DESIGN.md
+ * "Canonical score" (memory clause and SM/BW predicate of PAPER.md L87).
+ *
+ * Conventions
+ *  - Every function returns an int status: SCHED_OK (0) or a negative
+ *    SCHED_E_* code; sched_strerror() names it.  No C++ exception crosses
+ *    the ABI.  Output arguments are written only on SCHED_OK unless stated.
+ *  - Every input pointer is owned by the caller and may be freed as soon
+ *    as the call returns (sched_create copies the profile).
+ *  - A handle owns only host memory (and a small pinned staging buffer).
+ *    ALL device memory is caller-provided (d_workspace), and so is the
+ *    CUDA stream (cudaStream_t passed as void*; NULL = legacy default).
+ *  - A handle is not thread-safe; distinct handles are independent.
+ *  - Indices are uint64; the space must have |Omega| <= 2^63.
+ *  - Index order (R4): restricted-growth strings (RGS) of the partition in
+ *    lexicographic order; within a partition the level digits read as a
+ *    base-L number, most significant digit = client 0 (PER_CLIENT) or
+ *    group 0 (PER_GPU).  Ties between equal fp64 scores go to the lowest
+ *    index (BASELINE.json north_star).
+ */
+#ifndef SCHED_H_
+#define SCHED_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+  SCHED_OK = 0,
+  SCHED_E_INVALID = -1,     /* bad argument / profile / query */
+  SCHED_E_TOO_LARGE = -2,   /* |Omega| > 2^63, or tables exceed device limits */
+  SCHED_E_CUDA = -3,        /* a CUDA runtime call failed */
+  SCHED_E_CAPACITY = -4,    /* output/candidate capacity too small; *n_pareto = required */
+  SCHED_E_INFEASIBLE = -5,  /* no feasible configuration in the searched range
+                               (outputs ARE written, with valid = 0) */
+  SCHED_E_WORKSPACE = -6,   /* workspace too small or misaligned (256 B) */
+  SCHED_E_NODEVICE = -7     /* no CUDA device: there is no CPU fallback */
+};
+
+enum { SCHED_PER_CLIENT = 0, SCHED_PER_GPU = 1 };
+
+#define SCHED_MAX_WORKFLOWS 32
+#define SCHED_MAX_GPUS 16
+#define SCHED_MAX_PROFILE_LEVELS 32
+#define SCHED_MAX_SEARCH_LEVELS 8
+#define SCHED_MAX_WEIGHTS 8
+#define SCHED_MAX_EXPONENT 8
+#define SCHED_MAX_CLIENTS 48    /* MPS client limit */
+
+/* Offline solo + co-run profile (SM, memory, memory-bandwidth
+ * utilisation and average power per workflow task; Table II).
+ * Row-major; [N][L] means element (i, l) at i*L + l. */
+typedef struct {
+  int32_t n_workflows;          /* N_max >= 1: queue order = index order */
+  int32_t n_levels;             /* L_p >= 1: profile grid of MPS active-thread % */
+  const int32_t *level_pct;     /* [L_p] strictly ascending in (0,100]; must contain 100 */
+  const float *solo_time_s;     /* [N][L_p] > 0: solo wall time of the workflow at that level */
+  const float *solo_power_w;    /* [N][L_p] >= static_power_w: average GPU power */
+  const float *sm_util;         /* [N][L_p] >= 0: average SM utilisation, fraction of the GPU */
+  const float *bw_util;         /* [N][L_p] >= 0: average memory-BW utilisation, fraction */
+  const int32_t *max_mem_mib;   /* [N] >= 0: maximum memory of the task */
+  const float *corun_slowdown;  /* [N][L_p][N][L_p] >= 0: additive slowdown of i at level l
+                                   caused by co-runner j at level m; diagonal i == j ignored */
+  int32_t mem_capacity_mib;     /* device memory capacity (e.g. 81920 for A100X 80 GB) */
+  float static_power_w;         /* P_s > 0: static GPU power charged per busy second (R8, R9) */
+} sched_profile;
+
+/* One search request (queue, available GPUs, metric priority). */
+typedef struct {
+  int32_t n;                    /* search workflows [0, n), 1 <= n <= N_max */
+  int32_t g;                    /* available GPUs, 1..SCHED_MAX_GPUS */
+  int32_t max_clients;          /* C: MPS clients per GPU, 1..48; C >= n means uncapped */
+  uint32_t level_mask;          /* bit l selects profile level l for the search (L = popcount,
+                                   1..SCHED_MAX_SEARCH_LEVELS); digit d = d-th set bit */
+  int32_t level_scope;          /* SCHED_PER_CLIENT | SCHED_PER_GPU */
+  int32_t n_weights;            /* W, 0..SCHED_MAX_WEIGHTS */
+  const int32_t *weights;       /* [W][2] integer exponents (a,b) of F = X^a * Y^b,
+                                   0 <= a,b <= 8, a+b >= 1 */
+  uint64_t index_lo, index_hi;  /* searched window [lo, hi); hi = UINT64_MAX means |Omega| */
+  int32_t shard_rank;           /* this rank's share: chunks c with c % shard_count == rank */
+  int32_t shard_count;          /* >= 1 (multi-GPU split, one process per GPU) */
+  int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 10..40 (default 22) */
+  int32_t want_pareto;          /* nonzero: also compute the (T, E) Pareto set */
+  uint32_t candidate_cap;       /* device Pareto-candidate buffer records; 0 = 1<<20 */
+} sched_query;
+
+/* One configuration and its scores.  score64/x64/y64/makespan_s/energy_j are
+ * the fp64 canonical values (bitwise those of the CPU oracle); score32/x32/
+ * y32 are the fp32 hot-loop values of the same configuration. */
+typedef struct {
+  uint64_t index;
+  double score64, x64, y64;     /* F = X^a Y^b, X = T_seq/T, Y = E_seq/E */
+  double makespan_s, energy_j;  /* T, E of the configuration */
+  float score32, x32, y32;
+  int32_t valid;                /* 0: no feasible configuration found (pick is empty) */
+} sched_pick;
+
+typedef struct {
+  uint64_t n_configs;           /* configurations scored by this call (range x shard) */
+  uint64_t n_feasible;          /* of which memory-feasible */
+  uint64_t n_refined;           /* fp64 re-scores issued by the fp32 screen */
+  uint64_t n_candidates;        /* Pareto candidates emitted to the device buffer */
+  double t_seq_s, e_seq_j;      /* sequential baselines */
+  float search_ms;              /* device time of the search kernel(s) (CUDA events) */
+  float total_ms;               /* device time of the whole call on the stream */
+  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile kernel, 2 partition DFS kernel */
+  int32_t grid_ctas;            /* persistent CTAs launched by the search kernel */
+} sched_stats;
+
+typedef struct sched_handle sched_handle;
+
+/* Copy + validate the profile, precompute host-side derived tables.
+ * Errors: SCHED_E_INVALID (null/invalid field, p < P_s, level grid without 100). */
+int sched_create(const sched_profile *profile, sched_handle **out);
+int sched_destroy(sched_handle *h);
+
+/* Exact |Omega| of the query's full space (ignores index window and shard).
+ * Host only (no device needed).  SCHED_E_TOO_LARGE if > 2^63. */
+int sched_count(const sched_query *q, uint64_t *count);
+
+/* Bytes of device workspace sched_search needs for this query. */
+int sched_workspace_size(const sched_handle *h, const sched_query *q, size_t *bytes);
+
+/* Upload the query's staged tables (profile rows at the searched levels,
+ * DP count table) into d_workspace on `stream`.  Optional: sched_search
+ * stages itself when the workspace does not already hold this query. */
+int sched_stage(sched_handle *h, const sched_query *q, void *d_workspace, size_t ws_bytes,
+                void *cuda_stream);
+
+/* Exhaustive search of [index_lo, index_hi) restricted to this shard.
+ * best[W]: best configuration per weight (max F; ties -> lowest index).
+ * pareto[pareto_cap]: Pareto set of distinct (T,E) ordered by X descending,
+ * one (lowest) index per point; *n_pareto = its size (if > pareto_cap the
+ * call returns SCHED_E_CAPACITY and *n_pareto is the required size).
+ * Synchronous w.r.t. its host outputs (synchronises `stream`).
+ * stats may be NULL.  Errors: INVALID, TOO_LARGE, WORKSPACE, CUDA, CAPACITY,
+ * INFEASIBLE (outputs written with valid = 0), NODEVICE. */
+int sched_search(sched_handle *h, const sched_query *q, void *d_workspace, size_t ws_bytes,
+                 void *cuda_stream, sched_pick *best, sched_pick *pareto, uint64_t pareto_cap,
+                 uint64_t *n_pareto, sched_stats *stats);
+
+/* Merge per-rank results of sharded searches (exact, deterministic,
+ * independent of the rank count): rank_best is [n_ranks][n_weights];
+ * rank_pareto is the concatenation of each rank's Pareto list, rank r
+ * contributing rank_npareto[r] picks.  Host only.  Invalid picks are skipped. */
+int sched_merge(int32_t n_ranks, int32_t n_weights, const sched_pick *rank_best,
+                const sched_pick *rank_pareto, const uint64_t *rank_npareto,
+                sched_pick *best, sched_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto);
+
+/* index -> configuration: group_of[i] in 0..k-1 (RGS, group 0 holds
+ * workflow 0) and level_of[i] = searched-level digit (0..L-1) of workflow i
+ * (PER_GPU: the digit of its group).  Host only. */
+int sched_unrank(const sched_query *q, uint64_t index, int8_t *group_of, int8_t *level_of);
+
+/* configuration -> index (inverse of sched_unrank).  group_of must be an
+ * RGS; PER_GPU requires equal level_of within a group.  Host only. */
+int sched_rank(const sched_query *q, const int8_t *group_of, const int8_t *level_of,
+               uint64_t *index);
+
+/* fp64 canonical score of one configuration on the host, weight w (0..W-1;
+ * with W == 0 score64 = X).  out->valid = 0 if memory-infeasible.  Host only. */
+int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int32_t w,
+                sched_pick *out);
+
+const char *sched_strerror(int status);
+
+/* Library version string, e.g. "sched-b200 0.1 sm_100a". */
+const char *sched_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SCHED_H_ */

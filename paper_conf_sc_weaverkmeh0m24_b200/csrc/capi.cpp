@@ -1,0 +1,366 @@
+// capi.cpp -- the extern "C" boundary declared in include/sched.h.
+// Argument checking, handle/cache management, staging, result conversion.
+// No exception crosses the ABI (every entry point catches).
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstring>
+#include <new>
+
+#include "sched_internal.hpp"
+
+using namespace sched;
+
+struct sched_handle {
+  Profile P;
+  // cached DP space for the last query shape
+  int sp_key[5] = {-1, -1, -1, -1, -1};
+  Space sp;
+  // staged workspace state
+  const void *staged_ws = nullptr;
+  std::vector<unsigned char> staged_blob;
+  void *pinned = nullptr;
+  size_t pinned_bytes = 0;
+};
+
+namespace {
+
+int get_space(sched_handle *h, const Query &q, const Space **out) {
+  const int key[5] = {q.n, q.g, q.c, q.L, q.scope};
+  if (std::memcmp(key, h->sp_key, sizeof key) != 0) {
+    int st = build_space(q, &h->sp);
+    if (st) {
+      h->sp_key[0] = -1;
+      return st;
+    }
+    std::memcpy(h->sp_key, key, sizeof key);
+  }
+  *out = &h->sp;
+  return SCHED_OK;
+}
+
+int resolve(sched_handle *h, const sched_query *qin, Query *q, const Space **sp) {
+  int st = resolve_query_shape(qin, h->P.lp, q);
+  if (st) return st;
+  if (q->n > h->P.n) return SCHED_E_INVALID;
+  st = get_space(h, *q, sp);
+  if (st) return st;
+  if (q->hi == UINT64_MAX || q->hi > (*sp)->total) q->hi = (*sp)->total;
+  if (q->lo > q->hi) return SCHED_E_INVALID;
+  return SCHED_OK;
+}
+
+int need_device() {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n < 1) {
+    cudaGetLastError();
+    return SCHED_E_NODEVICE;
+  }
+  return SCHED_OK;
+}
+
+int do_stage(sched_handle *h, const DevParams &dp, const std::vector<unsigned char> &blob, void *ws,
+             void *stream) {
+  if (h->pinned_bytes < blob.size()) {
+    if (h->pinned) cudaFreeHost(h->pinned);
+    h->pinned = nullptr;
+    h->pinned_bytes = 0;
+    if (cudaHostAlloc(&h->pinned, blob.size() + 4096, cudaHostAllocDefault) != cudaSuccess) {
+      cudaGetLastError();
+      return SCHED_E_CUDA;
+    }
+    h->pinned_bytes = blob.size() + 4096;
+  }
+  int st = stage_tables(dp, blob, ws, h->pinned, stream);
+  if (st) return st;
+  h->staged_ws = ws;
+  h->staged_blob = blob;
+  return SCHED_OK;
+}
+
+void fill_pick(const Query &q, const DevParams &dp, int w, const BestRec &b, sched_pick *o) {
+  std::memset(o, 0, sizeof *o);
+  if (!b.valid) return;
+  o->valid = 1;
+  o->index = b.idx;
+  o->makespan_s = b.t;
+  o->energy_j = b.e;
+  o->x64 = dp.tseq / b.t;
+  o->y64 = dp.eseq / b.e;
+  o->score64 = b.f;
+  o->x32 = 1.f / b.t32;
+  o->y32 = 1.f / b.e32;
+  float s = 1.f;
+  for (int i = 0; i < q.wa[w]; i++) s *= o->x32;
+  for (int i = 0; i < q.wb[w]; i++) s *= o->y32;
+  o->score32 = s;
+}
+
+}  // namespace
+
+#define GUARD_BEGIN try {
+#define GUARD_END                 \
+  }                               \
+  catch (const std::bad_alloc &) { \
+    return SCHED_E_TOO_LARGE;     \
+  }                               \
+  catch (...) {                   \
+    return SCHED_E_INVALID;       \
+  }
+
+extern "C" {
+
+int sched_create(const sched_profile *profile, sched_handle **out) {
+  GUARD_BEGIN
+  if (!out) return SCHED_E_INVALID;
+  *out = nullptr;
+  sched_handle *h = new sched_handle();
+  int st = validate_profile(profile, &h->P);
+  if (st) {
+    delete h;
+    return st;
+  }
+  *out = h;
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_destroy(sched_handle *h) {
+  GUARD_BEGIN
+  if (!h) return SCHED_E_INVALID;
+  if (h->pinned) cudaFreeHost(h->pinned);
+  delete h;
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_count(const sched_query *qin, uint64_t *count) {
+  GUARD_BEGIN
+  if (!count) return SCHED_E_INVALID;
+  Query q;
+  int st = resolve_query_shape(qin, 32, &q);
+  if (st) return st;
+  Space sp;
+  st = build_space(q, &sp);
+  if (st) return st;
+  *count = sp.total;
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_workspace_size(const sched_handle *hc, const sched_query *qin, size_t *bytes) {
+  GUARD_BEGIN
+  if (!hc || !bytes) return SCHED_E_INVALID;
+  sched_handle *h = const_cast<sched_handle *>(hc);
+  Query q;
+  const Space *sp;
+  int st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = build_stage(h->P, q, *sp, &blob, &dp);
+  if (st) return st;
+  *bytes = workspace_bytes(dp, 0);
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_stage(sched_handle *h, const sched_query *qin, void *ws, size_t ws_bytes, void *stream) {
+  GUARD_BEGIN
+  if (!h || !ws) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  Query q;
+  const Space *sp;
+  st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = build_stage(h->P, q, *sp, &blob, &dp);
+  if (st) return st;
+  if (ws_bytes < workspace_bytes(dp, 0) || ((uintptr_t)ws & 255)) return SCHED_E_WORKSPACE;
+  return do_stage(h, dp, blob, ws, stream);
+  GUARD_END
+}
+
+int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_bytes, void *stream,
+                 sched_pick *best, sched_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto,
+                 sched_stats *stats) {
+  GUARD_BEGIN
+  if (!h || !ws) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  Query q;
+  const Space *sp;
+  st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  if (q.nw > 0 && !best) return SCHED_E_INVALID;
+  if (q.want_pareto && (!n_pareto || (pareto_cap > 0 && !pareto))) return SCHED_E_INVALID;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = build_stage(h->P, q, *sp, &blob, &dp);
+  if (st) return st;
+  if (ws_bytes < workspace_bytes(dp, 0) || ((uintptr_t)ws & 255)) return SCHED_E_WORKSPACE;
+  cudaEvent_t t0, t1;
+  if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess) return SCHED_E_CUDA;
+  cudaEventRecord(t0, (cudaStream_t)stream);
+  if (h->staged_ws != ws || h->staged_blob != blob) {
+    st = do_stage(h, dp, blob, ws, stream);
+    if (st) return st;
+  }
+  LaunchInfo info;
+  std::vector<BestRec> bres;
+  std::vector<CandRec> front;
+  uint64_t ctr[kCtrN];
+  st = launch_search(dp, ws, ws_bytes, stream, &info, &bres, &front, ctr);
+  cudaEventRecord(t1, (cudaStream_t)stream);
+  cudaEventSynchronize(t1);
+  float total_ms = 0.f;
+  cudaEventElapsedTime(&total_ms, t0, t1);
+  cudaEventDestroy(t0);
+  cudaEventDestroy(t1);
+  if (st && st != SCHED_E_CAPACITY) return st;
+  if (ctr[kCtrOverflow]) st = SCHED_E_CAPACITY;
+  for (int w = 0; w < q.nw; w++) fill_pick(q, dp, w, bres[w], &best[w]);
+  if (q.want_pareto) {
+    *n_pareto = front.size();
+    if (front.size() > pareto_cap) {
+      st = SCHED_E_CAPACITY;
+    } else {
+      for (size_t k = 0; k < front.size(); k++) {
+        sched_pick &o = pareto[k];
+        std::memset(&o, 0, sizeof o);
+        o.valid = 1;
+        o.index = front[k].idx;
+        o.makespan_s = front[k].t;
+        o.energy_j = front[k].e;
+        o.x64 = dp.tseq / front[k].t;
+        o.y64 = dp.eseq / front[k].e;
+        o.score64 = o.x64;  // Pareto picks: score = X (throughput)
+        o.x32 = 1.f / front[k].t32;
+        o.y32 = 1.f / front[k].e32;
+        o.score32 = o.x32;
+      }
+    }
+  } else if (n_pareto) {
+    *n_pareto = 0;
+  }
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->n_configs = ctr[kCtrConfigs];
+    stats->n_feasible = ctr[kCtrFeasible];
+    stats->n_refined = ctr[kCtrRefined];
+    stats->n_candidates = ctr[kCtrCand];
+    stats->t_seq_s = dp.tseq;
+    stats->e_seq_j = dp.eseq;
+    stats->search_ms = info.search_ms;
+    stats->total_ms = total_ms;
+    stats->kernel_path = info.path;
+    stats->grid_ctas = info.grid;
+  }
+  if (st) return st;
+  if (ctr[kCtrFeasible] == 0) return SCHED_E_INFEASIBLE;
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_merge(int32_t n_ranks, int32_t n_weights, const sched_pick *rank_best,
+                const sched_pick *rank_pareto, const uint64_t *rank_npareto, sched_pick *best,
+                sched_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto) {
+  GUARD_BEGIN
+  return merge_picks(n_ranks, n_weights, rank_best, rank_pareto, rank_npareto, best, pareto, pareto_cap,
+                     n_pareto);
+  GUARD_END
+}
+
+int sched_unrank(const sched_query *qin, uint64_t index, int8_t *group_of, int8_t *level_of) {
+  GUARD_BEGIN
+  if (!group_of || !level_of) return SCHED_E_INVALID;
+  Query q;
+  int st = resolve_query_shape(qin, 32, &q);
+  if (st) return st;
+  Space sp;
+  st = build_space(q, &sp);
+  if (st) return st;
+  int8_t dig[kMaxN];
+  int k;
+  st = host_unrank(sp, index, group_of, dig, &k);
+  if (st) return st;
+  for (int i = 0; i < q.n; i++) level_of[i] = q.scope == SCHED_PER_CLIENT ? dig[i] : dig[group_of[i]];
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_rank(const sched_query *qin, const int8_t *group_of, const int8_t *level_of, uint64_t *index) {
+  GUARD_BEGIN
+  if (!group_of || !level_of || !index) return SCHED_E_INVALID;
+  Query q;
+  int st = resolve_query_shape(qin, 32, &q);
+  if (st) return st;
+  Space sp;
+  st = build_space(q, &sp);
+  if (st) return st;
+  int8_t dig[kMaxN];
+  int k = 0;
+  for (int i = 0; i < q.n; i++) k = group_of[i] + 1 > k ? group_of[i] + 1 : k;
+  if (q.scope == SCHED_PER_CLIENT) {
+    for (int i = 0; i < q.n; i++) dig[i] = level_of[i];
+  } else {
+    for (int g = 0; g < k; g++) dig[g] = -1;
+    for (int i = 0; i < q.n; i++) {
+      const int g = group_of[i];
+      if (g < 0 || g >= kMaxG) return SCHED_E_INVALID;
+      if (dig[g] >= 0 && dig[g] != level_of[i]) return SCHED_E_INVALID;
+      dig[g] = level_of[i];
+    }
+  }
+  return host_rank(sp, group_of, dig, index);
+  GUARD_END
+}
+
+int sched_score(const sched_handle *hc, const sched_query *qin, uint64_t index, int32_t w, sched_pick *out) {
+  GUARD_BEGIN
+  if (!hc || !out) return SCHED_E_INVALID;
+  sched_handle *h = const_cast<sched_handle *>(hc);
+  Query q;
+  const Space *sp;
+  int st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  if (w < 0 || (q.nw > 0 && w >= q.nw) || (q.nw == 0 && w != 0)) return SCHED_E_INVALID;
+  int8_t a[kMaxN], dig[kMaxN];
+  int k;
+  st = host_unrank(*sp, index, a, dig, &k);
+  if (st) return st;
+  std::memset(out, 0, sizeof *out);
+  out->index = index;
+  double T, E, ts, es;
+  host_constants(h->P, q, &ts, &es);
+  if (!host_score(h->P, q, a, k, dig, &T, &E)) return SCHED_OK;  // valid = 0: infeasible
+  out->valid = 1;
+  out->makespan_s = T;
+  out->energy_j = E;
+  out->x64 = ts / T;
+  out->y64 = es / E;
+  const int ea = q.nw ? q.wa[w] : 1, eb = q.nw ? q.wb[w] : 0;
+  out->score64 = host_objective(ts, es, T, E, ea, eb);
+  return SCHED_OK;
+  GUARD_END
+}
+
+const char *sched_strerror(int s) {
+  switch (s) {
+    case SCHED_OK: return "ok";
+    case SCHED_E_INVALID: return "invalid argument";
+    case SCHED_E_TOO_LARGE: return "space or tables too large";
+    case SCHED_E_CUDA: return "CUDA runtime error";
+    case SCHED_E_CAPACITY: return "capacity too small";
+    case SCHED_E_INFEASIBLE: return "no feasible configuration";
+    case SCHED_E_WORKSPACE: return "workspace too small or misaligned";
+    case SCHED_E_NODEVICE: return "no CUDA device (no CPU fallback)";
+    default: return "unknown status";
+  }
+}
+
+const char *sched_version(void) { return "sched-b200 0.1 sm_100a"; }
+
+}  // extern "C"

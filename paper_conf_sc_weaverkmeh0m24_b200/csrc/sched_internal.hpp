@@ -1,0 +1,145 @@
+// sched_internal.hpp -- types shared by the host core (host_core.cpp), the
+// C ABI (capi.cpp) and the kernels (search.cu).  Not part of the public ABI.
+//
+// Citations: PAPER.md = /root/reference/PAPER.md; R<n> = DESIGN.md readings.
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+#include <vector>
+
+#include "sched.h"
+
+namespace sched {
+
+constexpr int kMaxN = SCHED_MAX_WORKFLOWS;      // 32
+constexpr int kMaxG = SCHED_MAX_GPUS;           // 16
+constexpr int kMaxL = SCHED_MAX_SEARCH_LEVELS;  // 8
+constexpr int kMaxW = SCHED_MAX_WEIGHTS;        // 8
+constexpr int kBuckets = 256;                   // Pareto staircase buckets (per warp)
+constexpr int kBucketShift = 18;                // 32 buckets per binade of T/T_seq
+constexpr uint16_t kNoState = 0xFFFF;
+constexpr int kUnitLog2 = 11;                   // generic kernel: 2048 configs per warp unit
+
+// Validated host copy of sched_profile.
+struct Profile {
+  int n = 0, lp = 0;
+  std::vector<int> pct;
+  std::vector<float> t, p, u, bw, d;  // [n][lp], d: [n][lp][n][lp]
+  std::vector<int> mem;
+  int mem_cap = 0;
+  float ps = 0.f;
+  int l100 = -1;
+};
+
+// Validated query (levels resolved to profile level indices).
+struct Query {
+  int n, g, c, L, scope, nw;
+  int lev[kMaxL];           // profile level index of searched digit d
+  int wa[kMaxW], wb[kMaxW];
+  uint64_t lo, hi;          // resolved window (hi <= |Omega|)
+  int rank, count, chunk_log2;
+  int want_pareto;
+  uint32_t cand_cap;
+};
+
+// DP count table (host + device): state = (elements placed, open groups,
+// histogram of non-full group sizes); W[s] = #(RGS completions x level
+// vectors) below s.  trans[s*tc + col]: col 0 = open a new group, col z =
+// join a group of size z (capped) / col 1 = join any group (uncapped).
+struct Space {
+  int n = 0, g = 0, c = 0, L = 0, scope = 0;
+  bool capped = false;
+  int tc = 0;
+  std::vector<uint64_t> W;
+  std::vector<uint16_t> trans;
+  int root = 0;
+  uint64_t total = 0;
+};
+
+// Device-side parameter block (kernel argument, by value).
+struct DevParams {
+  // problem
+  int n, g, c, L, scope, nw, capped, tc, R, ds;  // R = n*L rows, ds = d row stride
+  int wa[kMaxW], wb[kMaxW];
+  float delta[kMaxW];       // fp32 screen margin per weight
+  float gamma;              // Pareto "surely dominated" margin
+  float phat;               // P_s * T_seq / E_seq
+  double ps, tseq, eseq;
+  int mem_cap, want_pareto, root, nstates;
+  uint32_t bucket_base;     // (bits(T_lower) >> kBucketShift)
+  // work split
+  uint64_t lo, hi;          // window
+  uint64_t first_chunk;     // first owned chunk id
+  uint64_t n_owned;         // owned chunks intersecting [lo, hi)
+  int shard_count, chunk_log2, unit_log2;
+  uint64_t n_units;
+  // staged blob offsets (bytes from blob start) and size
+  uint32_t off_th, off_u, off_bw, off_dh, off_traw, off_praw, off_mem, off_d, off_W, off_trans;
+  uint32_t blob_bytes;
+  // workspace pointers
+  const unsigned char *blob;   // staged tables (device)
+  unsigned long long *ctr;     // counters (see kCtr*)
+  unsigned int *thr;           // [kMaxW] global fp32 proxy threshold bits (min)
+  unsigned int *stair;         // [kBuckets] raw staircase (float bits, min)
+  unsigned char *slots;        // [grid][W] BestRec
+  unsigned char *cand;         // [cand_cap] CandRec
+  uint32_t cand_cap;
+  unsigned char *out;          // finalize output area
+};
+
+enum {
+  kCtrUnit = 0,      // next work unit
+  kCtrCand = 1,      // candidates appended
+  kCtrConfigs = 2,   // configs scored
+  kCtrFeasible = 3,  // feasible configs
+  kCtrRefined = 4,   // fp64 refines
+  kCtrOverflow = 5,  // candidate overflow flag
+  kCtrSurv = 6,      // finalize: Pareto survivors
+  kCtrFront = 7,     // finalize: front size
+  kCtrN = 16
+};
+
+struct BestRec {      // 48 B
+  double f, t, e;
+  unsigned long long idx;
+  float t32, e32;     // normalised fp32 T/T_seq, E/E_seq of the hot loop
+  int valid, pad;
+};
+
+struct CandRec {      // 32 B
+  unsigned long long idx;
+  double t, e;
+  float t32, e32;
+};
+
+// ---- host core (host_core.cpp) ----
+int validate_profile(const sched_profile *in, Profile *out);
+int resolve_query(const Profile *P, const sched_query *q, Query *out, uint64_t *total);
+int resolve_query_shape(const sched_query *q, int n_profile_levels, Query *out);
+int build_space(const Query &q, Space *sp);
+int host_unrank(const Space &sp, uint64_t idx, int8_t *a, int8_t *digits, int *k);
+int host_rank(const Space &sp, const int8_t *a, const int8_t *digits, uint64_t *idx);
+void host_constants(const Profile &P, const Query &q, double *tseq, double *eseq);
+int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const int8_t *digits,
+               double *T, double *E);
+double host_objective(double tseq, double eseq, double T, double E, int a, int b);
+// staged table blob + DevParams (work split, bounds) for one query
+int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<unsigned char> *blob,
+                DevParams *dp);
+int merge_picks(int n_ranks, int nw, const sched_pick *rank_best, const sched_pick *rank_pareto,
+                const uint64_t *rank_np, sched_pick *best, sched_pick *pareto, uint64_t cap,
+                uint64_t *np);
+
+// ---- device launchers (search.cu) ----
+struct LaunchInfo {
+  int path, grid;
+  float search_ms;
+};
+size_t workspace_bytes(const DevParams &dp, int max_grid);
+int stage_tables(const DevParams &dp, const std::vector<unsigned char> &blob, void *d_ws, void *host_pinned,
+                 void *stream);
+int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, LaunchInfo *info,
+                  std::vector<BestRec> *best, std::vector<CandRec> *pareto, uint64_t *ctr_out);
+
+}  // namespace sched

@@ -1,0 +1,568 @@
+// search.cu -- the exhaustive configuration search on sm_100a.
+//
+//   k_generic   any scope / L / G / C / weights: per-lane unrank + successor
+//               walk, from-scratch fp32 group scoring, fp32 screens, fp64
+//               canonical refine of near-best / possibly-Pareto configurations.
+//   k_best_final, k_pareto_* : per-GPU finalize (exact best, exact Pareto).
+//
+// The method (PAPER.md L87 interference
+// predicate + memory clause, L91, L96 metrics, L116 product metric) is
+// evaluated in fp32 for every configuration; any configuration that could be
+// the best for some weight (within the proven fp32 error margin delta_w of
+// the running best) or could be on the Pareto front (not surely dominated by
+// a verified point) is re-scored in fp64 in the canonical order, so the
+// chosen indices and the Pareto set are bitwise those of the fp64 oracle.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+
+#include "device_common.cuh"
+#include "search_tile.cuh"
+
+namespace sched {
+
+// ------------------------------------------------------------ lane state
+struct LaneCfg {
+  int8_t a[kMaxN];
+  uint16_t st[kMaxN];   // st[i] = DP state after placing element i
+  uint32_t mask[kMaxG];
+  int8_t sz[kMaxG];
+  int k;
+  u64 v, Pn;            // level residue in [0, Pn), Pn = L^(#digits)
+  bool feasible;
+};
+
+__device__ __forceinline__ void cfg_feasibility(const Tables &tb, const DevParams &p, LaneCfg &c) {
+  bool ok = true;
+  for (int g = 0; g < c.k; g++) {
+    long long M = 0;
+    for (uint32_t mm = c.mask[g]; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
+    ok &= M <= (long long)p.mem_cap;
+  }
+  c.feasible = ok;
+}
+
+__device__ __forceinline__ int col_for(const DevParams &p, int j, int b, const int8_t *sz) {
+  if (j < b) {
+    if (p.capped) return sz[j] >= p.c ? -1 : sz[j];
+    return 1;
+  }
+  return b >= p.g ? -1 : 0;
+}
+
+__device__ __forceinline__ void place(LaneCfg &c, int i, int j) {
+  c.a[i] = (int8_t)j;
+  if (j == c.k) {
+    c.sz[c.k] = 0;
+    c.mask[c.k] = 0;
+    c.k++;
+  }
+  c.sz[j]++;
+  c.mask[j] |= 1u << i;
+}
+
+// index -> (RGS, residue) through the DP count table (R4 index order)
+__device__ bool dev_unrank(const Tables &tb, const DevParams &p, u64 idx, LaneCfg &c) {
+  u64 r = idx;
+  int s = p.root;
+  c.k = 0;
+  place(c, 0, 0);
+  c.st[0] = (uint16_t)s;
+  for (int i = 1; i < p.n; i++) {
+    int chosen = -1;
+    for (int j = 0; j <= c.k; j++) {
+      const int col = col_for(p, j, c.k, c.sz);
+      if (col < 0) {
+        if (j == c.k) break;
+        continue;
+      }
+      const uint16_t s2 = tb.trans[s * p.tc + col];
+      if (s2 == kNoState) continue;
+      const u64 w = tb.W[s2];
+      if (r < w) {
+        chosen = j;
+        s = s2;
+        break;
+      }
+      r -= w;
+    }
+    if (chosen < 0) return false;
+    place(c, i, chosen);
+    c.st[i] = (uint16_t)s;
+  }
+  c.Pn = tb.W[c.st[p.n - 1]];
+  c.v = r;
+  cfg_feasibility(tb, p, c);
+  return true;
+}
+
+// next RGS in lexicographic order (valid + completable), digits reset by caller
+__device__ bool dev_successor(const Tables &tb, const DevParams &p, LaneCfg &c) {
+  for (int i = p.n - 1; i >= 1; i--) {
+    const int j0 = c.a[i];
+    c.mask[j0] &= ~(1u << i);
+    if (--c.sz[j0] == 0) c.k--;
+    const int s = c.st[i - 1];
+    for (int j = j0 + 1; j <= c.k; j++) {
+      const int col = col_for(p, j, c.k, c.sz);
+      if (col < 0) {
+        if (j == c.k) break;
+        continue;
+      }
+      const uint16_t s2 = tb.trans[s * p.tc + col];
+      if (s2 == kNoState || tb.W[s2] == 0) continue;
+      place(c, i, j);
+      c.st[i] = s2;
+      for (int m = i + 1; m < p.n; m++) {  // greedy lexicographically-smallest completion
+        const int sm = c.st[m - 1];
+        for (int jj = 0; jj <= c.k; jj++) {
+          const int cl = col_for(p, jj, c.k, c.sz);
+          if (cl < 0) {
+            if (jj == c.k) break;
+            continue;
+          }
+          const uint16_t t2 = tb.trans[sm * p.tc + cl];
+          if (t2 == kNoState || tb.W[t2] == 0) continue;
+          place(c, m, jj);
+          c.st[m] = t2;
+          break;
+        }
+      }
+      return true;
+    }
+  }
+  return false;
+}
+
+__device__ __forceinline__ bool dev_advance(const Tables &tb, const DevParams &p, LaneCfg &c, u64 m) {
+  c.v += m;
+  while (c.v >= c.Pn) {
+    c.v -= c.Pn;
+    if (!dev_successor(tb, p, c)) return false;
+    c.Pn = tb.W[c.st[p.n - 1]];
+    cfg_feasibility(tb, p, c);
+  }
+  return true;
+}
+
+__device__ __forceinline__ void decode_levels(const DevParams &p, const LaneCfg &c, int *lam) {
+  const int nd = p.scope == SCHED_PER_CLIENT ? p.n : c.k;
+  int dig[kMaxN];
+  u64 x = c.v;
+  for (int d = nd - 1; d >= 0; d--) {
+    dig[d] = (int)(x % (u64)p.L);
+    x /= (u64)p.L;
+  }
+  for (int i = 0; i < p.n; i++) lam[i] = p.scope == SCHED_PER_CLIENT ? dig[i] : dig[c.a[i]];
+}
+
+// fp32 score, normalised: returns T/T_seq and E/E_seq (hot-loop precision)
+__device__ __forceinline__ void score32(const Tables &tb, const DevParams &p, const LaneCfg &c,
+                                        const int *lam, float &T, float &E) {
+  T = 0.f;
+  E = 0.f;
+  for (int g = 0; g < c.k; g++) {
+    const uint32_t m = c.mask[g];
+    float U = 0.f, B = 0.f, D = 0.f;
+    for (uint32_t mm = m; mm; mm &= mm - 1) {
+      const int i = __ffs(mm) - 1, r = i * p.L + lam[i];
+      U += tb.u[r];
+      B += tb.bw[r];
+      D += tb.dh[r];
+    }
+    const float cg = fmaxf(fmaxf(1.f, U), B);
+    float Tg = 0.f;
+    for (uint32_t mm = m; mm; mm &= mm - 1) {
+      const int i = __ffs(mm) - 1, ri = i * p.L + lam[i];
+      float s = 1.f;
+      for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) s += tb.d[ri * p.ds + (__ffs(m2) - 1) * p.L + lam[__ffs(m2) - 1]];
+      Tg = fmaxf(Tg, tb.th[ri] * s * cg);
+    }
+    T = fmaxf(T, Tg);
+    E += p.phat * Tg + D;
+  }
+}
+
+__device__ __forceinline__ float proxy(float T, float E, int a, int b) {
+  float q = 1.f;
+  for (int i = 0; i < a; i++) q *= T;
+  for (int i = 0; i < b; i++) q *= E;
+  return q;
+}
+
+// ------------------------------------------------------------ generic kernel
+constexpr int kThreads = 256;
+constexpr int kWarps = kThreads / 32;
+
+__global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  stage_blob(sm, p);
+  const Tables tb = tables_at(sm, p);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  float *pm = (float *)(sm + ((p.blob_bytes + 15) & ~15u)) + warp * kBuckets;
+  BestRec *red = (BestRec *)((float *)(sm + ((p.blob_bytes + 15) & ~15u)) + kWarps * kBuckets);
+
+  float thr[kMaxW];
+  BestRec lb[kMaxW];
+#pragma unroll
+  for (int w = 0; w < kMaxW; w++) {
+    thr[w] = __int_as_float(0x7f800000);
+    best_init(lb[w]);
+  }
+  u64 ncfg = 0, nfeas = 0, nref = 0;
+  const int ul = p.unit_log2, cl = p.chunk_log2;
+  LaneCfg c;
+  int lam[kMaxN];
+
+  for (;;) {
+    u64 unit = 0;
+    if (lane == 0) unit = atomicAdd(p.ctr + kCtrUnit, 1ull);
+    unit = __shfl_sync(0xffffffffu, unit, 0);
+    if (unit >= p.n_units) break;
+    const u64 ch = p.first_chunk + (unit >> (cl - ul)) * (u64)p.shard_count;
+    u64 s = (ch << cl) + ((unit & ((1ull << (cl - ul)) - 1)) << ul);
+    u64 e = s + (1ull << ul);
+    s = s > p.lo ? s : p.lo;
+    e = e < p.hi ? e : p.hi;
+    if (s >= e) continue;
+    // refresh shared thresholds and the staircase
+#pragma unroll
+    for (int w = 0; w < kMaxW; w++)
+      if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
+    if (p.want_pareto) refresh_stair(pm, p.stair);
+
+    u64 idx = s + lane;
+    if (idx < e && dev_unrank(tb, p, idx, c)) {
+      for (;;) {
+        ncfg++;
+        if (c.feasible) {
+          nfeas++;
+          decode_levels(p, c, lam);
+          float T, E;
+          score32(tb, p, c, lam, T, E);
+          bool need = false;
+          unsigned wneed = 0;
+#pragma unroll
+          for (int w = 0; w < kMaxW; w++) {
+            if (w < p.nw) {
+              const float q = proxy(T, E, p.wa[w], p.wb[w]);
+              thr[w] = fminf(thr[w], q);
+              if (q <= thr[w] * (1.f + p.delta[w])) {
+                need = true;
+                wneed |= 1u << w;
+              }
+            }
+          }
+          bool par = false;
+          if (p.want_pareto) par = !(E > pm[bucket_of(T, p.bucket_base)]);
+          if (need || par) {
+            nref++;
+            double T64, E64;
+            refine64(tb, p, c.mask, c.k, lam, &T64, &E64);
+#pragma unroll
+            for (int w = 0; w < kMaxW; w++) {
+              if (wneed >> w & 1u) {
+                const double F = objective64(p, T64, E64, p.wa[w], p.wb[w]);
+                if (!lb[w].valid || better(F, idx, lb[w].f, lb[w].idx)) {
+                  lb[w].f = F;
+                  lb[w].idx = idx;
+                  lb[w].t = T64;
+                  lb[w].e = E64;
+                  lb[w].t32 = T;
+                  lb[w].e32 = E;
+                  lb[w].valid = 1;
+                }
+              }
+            }
+            if (par) emit_candidate(p, pm, idx, T64, E64, T, E);
+          }
+        }
+        idx += 32;
+        if (idx >= e) break;
+        if (!dev_advance(tb, p, c, 32)) break;
+      }
+    }
+    __syncwarp();
+    // publish thresholds (warp min, one atomic per weight)
+#pragma unroll
+    for (int w = 0; w < kMaxW; w++) {
+      if (w < p.nw) {
+        float t = thr[w];
+#pragma unroll
+        for (int o = 16; o; o >>= 1) t = fminf(t, __shfl_xor_sync(0xffffffffu, t, o));
+        thr[w] = t;
+        if (lane == 0 && t < __uint_as_float(__ldcg(p.thr + w))) atomicMin(p.thr + w, __float_as_uint(t));
+      }
+    }
+  }
+  // ---- reductions: counters, per-CTA best slots ----
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    ncfg += __shfl_xor_sync(0xffffffffu, ncfg, o);
+    nfeas += __shfl_xor_sync(0xffffffffu, nfeas, o);
+    nref += __shfl_xor_sync(0xffffffffu, nref, o);
+  }
+  if (lane == 0) {
+    atomicAdd(p.ctr + kCtrConfigs, ncfg);
+    atomicAdd(p.ctr + kCtrFeasible, nfeas);
+    atomicAdd(p.ctr + kCtrRefined, nref);
+  }
+#pragma unroll
+  for (int w = 0; w < kMaxW; w++) {
+    if (w < p.nw) {
+      warp_best(lb[w]);
+      if (lane == 0) red[warp * kMaxW + w] = lb[w];
+    }
+  }
+  __syncthreads();
+  if (threadIdx.x < p.nw) {
+    const int w = threadIdx.x;
+    BestRec b = red[w];
+    for (int k = 1; k < kWarps; k++) {
+      const BestRec x = red[k * kMaxW + w];
+      if (x.valid && (!b.valid || better(x.f, x.idx, b.f, b.idx))) b = x;
+    }
+    ((BestRec *)p.slots)[(size_t)blockIdx.x * p.nw + w] = b;
+  }
+}
+
+// ------------------------------------------------------------ init / finalize
+__global__ void k_init(const DevParams p) {
+  const int t = threadIdx.x;
+  if (t < kCtrN) p.ctr[t] = 0ull;
+  if (t < kMaxW) p.thr[t] = 0x7f800000u;
+  for (int i = t; i < kBuckets; i += blockDim.x) p.stair[i] = 0x7f800000u;
+}
+
+// best per weight over the per-CTA slots -> out[0 .. W)
+__global__ void k_best_final(const DevParams p, int nslots) {
+  __shared__ BestRec red[32];
+  const int w = blockIdx.x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  BestRec b;
+  best_init(b);
+  for (int s = threadIdx.x; s < nslots; s += blockDim.x) {
+    const BestRec x = ((const BestRec *)p.slots)[(size_t)s * p.nw + w];
+    if (x.valid && (!b.valid || better(x.f, x.idx, b.f, b.idx))) b = x;
+  }
+  warp_best(b);
+  if (lane == 0) red[warp] = b;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int k = 1; k < (int)(blockDim.x >> 5); k++) {
+      const BestRec x = red[k];
+      if (x.valid && (!b.valid || better(x.f, x.idx, b.f, b.idx))) b = x;
+    }
+    ((BestRec *)p.out)[w] = b;
+  }
+}
+
+// Pareto finalize, stage 1: drop candidates surely (strictly) dominated by a
+// verified point of the final global staircase; compact survivors.
+__global__ void k_pareto_prefilter(const DevParams p, int ncand, unsigned int *surv) {
+  __shared__ float pm[kBuckets];
+  if (threadIdx.x < 32) refresh_stair(pm, p.stair);
+  __syncthreads();
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
+    const CandRec c = ((const CandRec *)p.cand)[i];
+    const float tl = __double2float_rd(__ddiv_rd(c.t, p.tseq));
+    const float el = __double2float_rd(__ddiv_rd(c.e, p.eseq));
+    const bool dom = el > pm[bucket_of(tl, p.bucket_base)];
+    if (!dom) {
+      const unsigned int k = (unsigned int)atomicAdd(p.ctr + kCtrSurv, 1ull);
+      surv[k] = (unsigned int)i;
+    }
+  }
+}
+
+// stage 2: exact O(m^2) dominance among survivors (smem tiles); keep[s] = 1 if
+// on the front (one representative per distinct (T,E): the lowest index).
+__global__ void k_pareto_exact(const DevParams p, const unsigned int *surv, unsigned int *keep) {
+  __shared__ CandRec tile[256];
+  const int m = (int)(*(volatile unsigned long long *)(p.ctr + kCtrSurv));
+  const CandRec *cand = (const CandRec *)p.cand;
+  for (int base = blockIdx.x * blockDim.x; base < m; base += gridDim.x * blockDim.x) {
+    const int s = base + threadIdx.x;
+    CandRec me;
+    if (s < m) me = cand[surv[s]];
+    bool alive = s < m;
+    for (int t0 = 0; t0 < m; t0 += 256) {
+      __syncthreads();
+      if (t0 + threadIdx.x < m) tile[threadIdx.x] = cand[surv[t0 + threadIdx.x]];
+      __syncthreads();
+      const int nt = min(256, m - t0);
+      if (alive) {
+        for (int k = 0; k < nt; k++) {
+          const CandRec o = tile[k];
+          const bool dom = (o.t <= me.t && o.e <= me.e && (o.t < me.t || o.e < me.e)) ||
+                           (o.t == me.t && o.e == me.e && (o.idx < me.idx || (o.idx == me.idx && t0 + k < s)));
+          if (dom) {
+            alive = false;
+            break;
+          }
+        }
+      }
+    }
+    if (s < m) keep[s] = alive ? 1u : 0u;
+  }
+}
+
+// stage 3: order the front by T ascending (= X descending) into out[W ...]
+__global__ void k_pareto_order(const DevParams p, const unsigned int *surv, const unsigned int *keep,
+                               int out_cap) {
+  const int m = (int)(*(volatile unsigned long long *)(p.ctr + kCtrSurv));
+  const CandRec *cand = (const CandRec *)p.cand;
+  CandRec *out = (CandRec *)(p.out + sizeof(BestRec) * kMaxW);
+  for (int s = blockIdx.x * blockDim.x + threadIdx.x; s < m; s += gridDim.x * blockDim.x) {
+    if (!keep[s]) continue;
+    const CandRec me = cand[surv[s]];
+    int rank = 0;
+    for (int t = 0; t < m; t++)
+      if (keep[t] && cand[surv[t]].t < me.t) rank++;
+    if (rank < out_cap) out[rank] = me;
+    atomicAdd(p.ctr + kCtrFront, 1ull);
+  }
+}
+
+// ------------------------------------------------------------ launcher
+namespace {
+constexpr int kMaxGrid = 4096;
+constexpr int kFrontCap = 1 << 16;
+
+struct WsLayout {
+  size_t ctr, thr, stair, blob, slots, cand, surv, keep, out, total;
+};
+
+WsLayout layout(const DevParams &dp) {
+  WsLayout L;
+  size_t o = 0;
+  auto take = [&](size_t b) {
+    o = (o + 255) / 256 * 256;
+    size_t r = o;
+    o += b;
+    return r;
+  };
+  L.ctr = take(8 * kCtrN);
+  L.thr = take(4 * kMaxW);
+  L.stair = take(4 * kBuckets);
+  L.blob = take(dp.blob_bytes);
+  L.slots = take(sizeof(BestRec) * kMaxW * (size_t)kMaxGrid);
+  L.cand = take(sizeof(CandRec) * (size_t)dp.cand_cap);
+  L.surv = take(4 * (size_t)dp.cand_cap);
+  L.keep = take(4 * (size_t)dp.cand_cap);
+  L.out = take(sizeof(BestRec) * kMaxW + sizeof(CandRec) * (size_t)kFrontCap);
+  L.total = (o + 255) / 256 * 256;
+  return L;
+}
+}  // namespace
+
+size_t workspace_bytes(const DevParams &dp, int) { return layout(dp).total; }
+
+#define CK(x)                                   \
+  do {                                          \
+    cudaError_t e_ = (x);                       \
+    if (e_ != cudaSuccess) return SCHED_E_CUDA; \
+  } while (0)
+
+int stage_tables(const DevParams &dp, const std::vector<unsigned char> &blob, void *d_ws, void *host_pinned,
+                 void *stream) {
+  const WsLayout L = layout(dp);
+  cudaStream_t st = (cudaStream_t)stream;
+  unsigned char *ws = (unsigned char *)d_ws;
+  const void *src = blob.data();
+  if (host_pinned) {
+    std::memcpy(host_pinned, blob.data(), blob.size());
+    src = host_pinned;
+  }
+  CK(cudaMemcpyAsync(ws + L.blob, src, blob.size(), cudaMemcpyHostToDevice, st));
+  return SCHED_OK;
+}
+
+int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, LaunchInfo *info,
+                  std::vector<BestRec> *best, std::vector<CandRec> *pareto, uint64_t *ctr_out) {
+  const WsLayout L = layout(dp);
+  if (ws_bytes < L.total || ((uintptr_t)d_ws & 255)) return SCHED_E_WORKSPACE;
+  unsigned char *ws = (unsigned char *)d_ws;
+  cudaStream_t st = (cudaStream_t)stream;
+  dp.blob = ws + L.blob;
+  dp.ctr = (unsigned long long *)(ws + L.ctr);
+  dp.thr = (unsigned int *)(ws + L.thr);
+  dp.stair = (unsigned int *)(ws + L.stair);
+  dp.slots = ws + L.slots;
+  dp.cand = ws + L.cand;
+  dp.out = ws + L.out;
+  int dev = 0, nsm = 0;
+  CK(cudaGetDevice(&dev));
+  CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+
+  cudaEvent_t e0, e1, e2;
+  CK(cudaEventCreate(&e0));
+  CK(cudaEventCreate(&e1));
+  CK(cudaEventCreate(&e2));
+  CK(cudaEventRecord(e0, st));
+  k_init<<<1, 256, 0, st>>>(dp);
+  CK(cudaGetLastError());
+
+  int grid = 0, path = 0;
+  TileLaunch tl;
+  if (tile_eligible(dp, &tl)) {
+    path = 1;
+    CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid));
+  } else {
+    const size_t smem = ((dp.blob_bytes + 15) & ~15u) + sizeof(float) * kWarps * kBuckets +
+                        sizeof(BestRec) * kWarps * kMaxW;
+    CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_generic, kThreads, smem));
+    if (occ < 1) return SCHED_E_TOO_LARGE;
+    grid = std::min(kMaxGrid, nsm * occ);
+    CK(cudaEventRecord(e1, st));
+    k_generic<<<grid, kThreads, smem, st>>>(dp);
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(e2, st));
+  }
+  // finalize
+  if (dp.nw > 0) {
+    k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid);
+    CK(cudaGetLastError());
+  }
+  uint64_t ctr[kCtrN];
+  CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  int ncand = (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap);
+  if (dp.want_pareto && ncand > 0) {
+    unsigned int *surv = (unsigned int *)(ws + L.surv), *keep = (unsigned int *)(ws + L.keep);
+    k_pareto_prefilter<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, ncand, surv);
+    CK(cudaGetLastError());
+    k_pareto_exact<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, surv, keep);
+    CK(cudaGetLastError());
+    k_pareto_order<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, surv, keep,
+                                                                                        kFrontCap);
+    CK(cudaGetLastError());
+  }
+  CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
+  best->resize(kMaxW);
+  CK(cudaMemcpyAsync(best->data(), dp.out, sizeof(BestRec) * kMaxW, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  const uint64_t nfront = dp.want_pareto && ncand > 0 ? ctr[kCtrFront] : 0;
+  pareto->resize(std::min<uint64_t>(nfront, kFrontCap));
+  if (!pareto->empty()) {
+    CK(cudaMemcpyAsync(pareto->data(), dp.out + sizeof(BestRec) * kMaxW, sizeof(CandRec) * pareto->size(),
+                       cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  float ms = 0.f;
+  CK(cudaEventElapsedTime(&ms, e1, e2));
+  info->search_ms = ms;
+  info->grid = grid;
+  info->path = path;
+  for (int k = 0; k < kCtrN; k++) ctr_out[k] = ctr[k];
+  ctr_out[kCtrFront] = nfront;
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaEventDestroy(e2);
+  if (nfront > kFrontCap) return SCHED_E_CAPACITY;
+  return SCHED_OK;
+}
+
+}  // namespace sched

@@ -1,0 +1,148 @@
+"""C-ABI library: loads, exports every symbol of include/sched.h, and its
+host-side logic (count, unrank/rank, fp64 score, merge, validation) agrees
+with the oracle.  No device compute (runs without a GPU)."""
+import ctypes as C
+import os
+import random
+import re
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_weaverkmeh0m24_b200 as S
+from paper_conf_sc_weaverkmeh0m24_b200 import build as B
+from synth import CONFIGS, config, make_profile, Query, PER_CLIENT, PER_GPU
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def built():
+    B.build()
+
+
+def test_exports_match_header():
+    hdr = open(os.path.join(ROOT, "include", "sched.h")).read()
+    decl = set(re.findall(r"^\s*(?:int|const char \*)\s*(sched_\w+)\s*\(", hdr, re.M))
+    assert decl == set(S.EXPORTS)
+    lib = C.CDLL(S.sched.SO_PATH)
+    for name in decl:
+        assert hasattr(lib, name), name
+
+
+def test_so_is_sm100a():
+    out = os.popen(f"/usr/local/cuda/bin/cuobjdump --list-elf {S.sched.SO_PATH}").read()
+    assert "sm_100a" in out
+
+
+@pytest.mark.parametrize("name", list(CONFIGS))
+def test_count_unrank_rank_match_oracle(name):
+    prof, q = config(name)
+    tot = S.count(q)
+    assert tot == oracle.count(q)
+    rnd = random.Random(hash(name) & 0xffff)
+    for idx in [0, 1, tot - 1, tot // 2] + [rnd.randrange(tot) for _ in range(40)]:
+        a, lv = S.unrank(q, idx)
+        oa, od = oracle.config(q, idx)
+        assert a == oa
+        assert lv == [od[i] if q.scope == PER_CLIENT else od[oa[i]] for i in range(q.n)]
+        assert S.rank(q, a, lv) == idx
+
+
+def test_unrank_bijection_small():
+    for (n, g, c, L, sc) in [(5, 3, 2, 2, PER_GPU), (4, 2, 4, 2, PER_CLIENT), (6, 4, 3, 3, PER_GPU),
+                             (7, 7, 7, 1, PER_GPU), (6, 2, 3, 2, PER_CLIENT)]:
+        q = Query(n, g, c, tuple(range(L)), sc, ())
+        tot = S.count(q)
+        prev = None
+        for idx in range(tot):
+            a, lv = S.unrank(q, idx)
+            assert S.rank(q, a, lv) == idx
+            key = (tuple(a), tuple(lv[i] for i in range(n)) if sc == PER_CLIENT else
+                   tuple(lv[a.index(b)] for b in range(max(a) + 1)))
+            assert prev is None or key > prev      # strictly increasing (R4)
+            prev = key
+
+
+def test_count_too_large():
+    q = Query(16, 8, 16, (0, 1, 2, 3), PER_CLIENT, ())
+    with pytest.raises(S.SchedError) as e:
+        S.count(q)
+    assert e.value.status == S.sched.SCHED_E_TOO_LARGE
+
+
+@pytest.mark.parametrize("name", ["c1", "c3", "c4", "c5"])
+def test_host_score_bitwise_oracle(name):
+    prof, q = config(name)
+    sch = S.Scheduler(prof)
+    tot = S.count(q)
+    rnd = random.Random(5)
+    ts, es = oracle.constants(prof, q)
+    for idx in [0, tot - 1] + [rnd.randrange(tot) for _ in range(30)]:
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, idx))
+        for w, (a, b) in enumerate(q.weights):
+            p = sch.score(q, idx, w)
+            assert p.valid == ok
+            if ok:
+                assert p.makespan_s == T and p.energy_j == E
+                assert p.score64 == oracle.objective(ts, es, T, E, a, b)
+
+
+def test_invalid_profiles_rejected():
+    prof = make_profile(4, levels=(50, 100), seed=1)
+    bad = make_profile(4, levels=(50, 100), seed=1)
+    bad.solo_power_w[0, 0] = 10.0            # below static power
+    with pytest.raises(S.SchedError):
+        S.Scheduler(bad)
+    bad = make_profile(4, levels=(50, 100), seed=1)
+    bad.level_pct = np.array([25, 50], np.int32)   # no 100% column
+    with pytest.raises(S.SchedError):
+        S.Scheduler(bad)
+    sch = S.Scheduler(prof)
+    for q in [Query(5, 2, 4, (50, 100), PER_GPU, ()), Query(4, 0, 4, (50, 100), PER_GPU, ()),
+              Query(4, 2, 4, (50, 100), PER_GPU, ((0, 0),)), Query(4, 2, 4, (50, 100), 3, ())]:
+        with pytest.raises(S.SchedError):
+            sch.workspace_size(q)
+
+
+def test_merge_host():
+    """sched_merge against a brute-force merge of random per-rank records."""
+    rnd = random.Random(3)
+    R, W = 4, 3
+    rank_best, rank_par = [], []
+    allpts = []
+    for r in range(R):
+        bl = []
+        for w in range(W):
+            p = S.Pick()
+            p.valid = rnd.random() < 0.8
+            p.index = rnd.randrange(1000)
+            p.score64 = rnd.choice([1.0, 1.5, 2.0])
+            bl.append(p)
+        rank_best.append(bl)
+        pl = []
+        for _ in range(rnd.randrange(6)):
+            p = S.Pick()
+            p.valid = 1
+            p.index = rnd.randrange(1000)
+            p.makespan_s = rnd.choice([1.0, 2.0, 3.0])
+            p.energy_j = rnd.choice([1.0, 2.0, 3.0])
+            pl.append(p)
+            allpts.append((p.makespan_s, p.energy_j, p.index))
+        rank_par.append(pl)
+    best, par = S.merge(rank_best, rank_par, W)
+    for w in range(W):
+        cands = [rank_best[r][w] for r in range(R) if rank_best[r][w].valid]
+        if not cands:
+            assert not best[w].valid
+            continue
+        exp = max(cands, key=lambda p: (p.score64, -p.index))
+        assert (best[w].index, best[w].score64) == (exp.index, exp.score64)
+    front = {}
+    for t, e, i in allpts:
+        if any((t2 <= t and e2 <= e and (t2 < t or e2 < e)) for t2, e2, _ in allpts):
+            continue
+        front[(t, e)] = min(i, front.get((t, e), i))
+    exp = sorted([(t, e, i) for (t, e), i in front.items()])
+    assert [(p.makespan_s, p.energy_j, p.index) for p in par] == exp

@@ -1,0 +1,172 @@
+"""GPU parity: the CUDA search (through the C ABI) against the CPU oracle.
+
+Bar (BASELINE.json north_star): configuration counts, chosen indices (ties
+-> lowest index) and the Pareto set bit-exact; the fp64 scores of the picks
+bitwise equal to the oracle's; the fp32 hot-loop scores within 1e-5
+relative of the oracle's fp64.
+"""
+import random
+
+import pytest
+
+import oracle
+import paper_conf_sc_weaverkmeh0m24_b200 as S
+from synth import CONFIGS, config, make_profile, Query, PER_CLIENT, PER_GPU
+
+pytestmark = pytest.mark.gpu
+
+REL32 = 1e-5
+
+
+def check(res, ref, q, sched=None):
+    nw = len(q.weights)
+    for w in range(nw):
+        r = ref["best"][w]
+        b = res.best[w]
+        if r is None:
+            assert not b.valid
+            continue
+        assert b.valid
+        assert b.index == r[0], (w, b.index, r)
+        assert b.score64 == r[1] and b.makespan_s == r[2] and b.energy_j == r[3]
+        assert abs(b.score32 / r[1] - 1) <= REL32
+        assert abs(b.x32 / (ref["tseq"] / r[2]) - 1) <= REL32
+        assert abs(b.y32 / (ref["eseq"] / r[3]) - 1) <= REL32
+    if q.want_pareto:
+        got = [(p.index, p.makespan_s, p.energy_j) for p in res.pareto]
+        assert got == ref["pareto"]
+        for p in res.pareto:
+            assert abs(p.x32 / (ref["tseq"] / p.makespan_s) - 1) <= REL32
+            assert abs(p.y32 / (ref["eseq"] / p.energy_j) - 1) <= REL32
+    assert res.stats["n_configs"] == ref["nconfigs"]
+    assert res.stats["n_feasible"] == ref["nfeasible"]
+
+
+def _cases():
+    rnd = random.Random(2024)
+    out = []
+    for t in range(40):
+        n = rnd.randint(2, 8)
+        g = rnd.randint(1, 5)
+        c = rnd.randint(max(1, -(-n // g)), n)
+        L = rnd.randint(1, 4)
+        levels = tuple(sorted(rnd.sample([25, 50, 75, 100], L)))
+        scope = rnd.choice([PER_CLIENT, PER_GPU])
+        if scope == PER_CLIENT and L ** n > 5000:
+            scope = PER_GPU
+        ws = tuple(rnd.sample([(1, 0), (0, 1), (1, 1), (2, 1), (1, 2), (3, 1), (1, 3), (4, 4)],
+                              rnd.randint(0, 5)))
+        out.append((t, n, g, c, levels, scope, ws))
+    return out
+
+
+@pytest.mark.parametrize("t,n,g,c,levels,scope,ws", _cases())
+def test_small_spaces_full(t, n, g, c, levels, scope, ws):
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=500 + t)
+    q = Query(n, g, c, levels, scope, ws, True)
+    ref = oracle.search(prof, q)
+    res = S.Scheduler(prof).search(q)
+    check(res, ref, q)
+
+
+def test_c1_full():
+    prof, q = config("c1")
+    check(S.Scheduler(prof).search(q), oracle.search(prof, q), q)
+
+
+def test_c2_full():
+    prof, q = config("c2")
+    q2 = Query(q.n, q.g, q.c, q.levels, q.scope, ((1, 0), (1, 1), (0, 1)), True)
+    ref = oracle.search_parallel(prof, q2)
+    check(S.Scheduler(prof).search(q2), ref, q2)
+
+
+def _windows(tot, chunk, rnd, size):
+    ws = [(0, size), (tot - size, tot), (chunk - size // 2, chunk + size // 2),
+          (3 * chunk - 7, 3 * chunk + size - 7)]
+    ws += [(x, x + size) for x in (rnd.randrange(tot - size) for _ in range(4))]
+    return ws
+
+
+@pytest.mark.parametrize("name", ["c3", "c4", "c5"])
+def test_windows_big_spaces(name):
+    prof, q = config(name)
+    tot = S.count(q)
+    sch = S.Scheduler(prof)
+    rnd = random.Random(11)
+    for lo, hi in _windows(tot, 1 << 22, rnd, 300_000):
+        qw = q.with_range(lo, hi)
+        check(sch.search(qw), oracle.search(prof, qw), qw)
+
+
+@pytest.mark.parametrize("R", [2, 3, 8])
+def test_sharded_merge_equals_single(R):
+    prof, q = config("c4")
+    q = Query(q.n, q.g, q.c, q.levels, q.scope, ((1, 1), (2, 1), (1, 0)), True)
+    lo = 123_456_789_000
+    qw = q.with_range(lo, lo + 5 * (1 << 16) + 333)
+    sch = S.Scheduler(prof)
+    one = sch.search(qw, chunk_log2=16)
+    bests, pars, ncfg = [], [], 0
+    for r in range(R):
+        res = sch.search(qw, shard=(r, R), chunk_log2=16)
+        bests.append(res.best)
+        pars.append(res.pareto)
+        ncfg += res.stats["n_configs"]
+    mb, mp = S.merge(bests, pars, 3)
+    assert ncfg == one.stats["n_configs"] == qw.index_hi - qw.index_lo
+    assert [b.index for b in mb] == [b.index for b in one.best]
+    assert [b.score64 for b in mb] == [b.score64 for b in one.best]
+    assert [(p.index, p.makespan_s, p.energy_j) for p in mp] == \
+        [(p.index, p.makespan_s, p.energy_j) for p in one.pareto]
+    check(one, oracle.search(prof, qw), qw)
+
+
+def test_edge_cases():
+    prof = make_profile(6, levels=(50, 100), seed=77)
+    sch = S.Scheduler(prof)
+    # empty window
+    q = Query(6, 3, 6, (50, 100), PER_GPU, ((1, 1),), True, 10, 10)
+    res = sch.search(q)
+    assert res.stats["n_configs"] == 0 and res.status == S.sched.SCHED_E_INFEASIBLE
+    # single configuration space: G = 1, one level
+    q = Query(6, 1, 6, (100,), PER_GPU, ((1, 0), (0, 1)), True)
+    check(sch.search(q), oracle.search(prof, q), q)
+    # n = 1
+    q = Query(1, 4, 1, (50, 100), PER_CLIENT, ((1, 1),), True)
+    check(sch.search(q), oracle.search(prof, q), q)
+    # all infeasible: two WarpX must share one GPU
+    p2 = make_profile(3, levels=(100,), seed=1, archetypes=[11, 12, 11])
+    q = Query(3, 1, 3, (100,), PER_GPU, ((1, 1),), True)
+    res = S.Scheduler(p2).search(q)
+    assert res.status == S.sched.SCHED_E_INFEASIBLE and not res.best[0].valid and res.pareto == []
+    # ragged window inside a partition
+    q = Query(6, 3, 6, (50, 100), PER_CLIENT, ((2, 1), (1, 2)), True, 37, 1001)
+    check(sch.search(q), oracle.search(prof, q), q)
+
+
+def test_c3_full_size_properties():
+    """Full c3 (2.6e10 configs) in the bench launch configuration; the oracle
+    checks the picks one by one and bounds them with random windows."""
+    prof, q = config("c3")
+    sch = S.Scheduler(prof)
+    res = sch.search(q)
+    tot = S.count(q)
+    assert res.stats["n_configs"] == tot
+    ts, es = oracle.constants(prof, q)
+    b = res.best[0]
+    ok, T, E = oracle.score(prof, q, *oracle.config(q, b.index))
+    assert ok and b.makespan_s == T and b.energy_j == E
+    assert b.score64 == oracle.objective(ts, es, T, E, 1, 1)
+    for p in res.pareto:
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
+        assert ok and (T, E) == (p.makespan_s, p.energy_j)
+    front = [(p.makespan_s, p.energy_j) for p in res.pareto]
+    rnd = random.Random(5)
+    for _ in range(6):
+        lo = rnd.randrange(tot - 200_000)
+        r = oracle.search(prof, q.with_range(lo, lo + 200_000))
+        if r["best"][0] is not None:
+            assert r["best"][0][1] < b.score64 or (r["best"][0][1] == b.score64 and r["best"][0][0] >= b.index)
+        for _, T, E in r["pareto"]:
+            assert any(t2 <= T and e2 <= E for t2, e2 in front)
