@@ -70,39 +70,72 @@ __device__ __forceinline__ void stage_blob(unsigned char *sm, const DevParams &p
 }
 
 // --------------------------------------------------------------- staircase
-// bucket of a positive normalised makespan (monotone non-decreasing in v)
-__device__ __forceinline__ int bucket_of(float v, uint32_t base) {
-  const int b = (int)(__float_as_uint(v) >> kBucketShift) - (int)base;
+// Sound Pareto screen.  Verified (fp64) points p
+// are keyed by their EXACT canonical makespan T_p (buckets of the fp64 bits
+// of T, monotone) and carry val_p = up(E_p/E_seq * (1+gamma)) >= the fp32
+// error band of any E.  A configuration with exact T and fp32 Ehat is
+// dominated by p if T >= T_p and Ehat > val_p (then E > E_p exactly):
+//   pm[j] = min val over points in buckets < j        (T > T_p for sure)
+//   bp[j] = min (val << 32 | slot) over points in bucket j; the point's
+//           exact T is read back from the candidate buffer slot.
+// Equal-T ties (configurations sharing a bottleneck group) are therefore
+// screened exactly.  All updates are monotone minima (race-free merges).
+struct Stair {
+  unsigned int *pm;
+  unsigned long long *bp;
+};
+
+__device__ __forceinline__ int bucket_of(double T, uint32_t base) {
+  const int b = (int)((unsigned long long)__double_as_longlong(T) >> kBucketShift) - (int)base;
   return b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
 }
 
-// Per-warp exclusive prefix-min of the global raw staircase:
-// pm[i] = min_{j<i} raw[j].  All 32 lanes must call.
-__device__ __forceinline__ void refresh_stair(float *pm, const unsigned int *raw) {
+__device__ __forceinline__ void stair_init(Stair s) {
+  for (int i = threadIdx.x; i < kBuckets; i += blockDim.x) {
+    s.pm[i] = 0x7f800000u;
+    s.bp[i] = ~0ull;
+  }
+}
+
+// Warp-cooperative merge of the global staircase into a CTA staircase.
+__device__ __forceinline__ void stair_merge(Stair s, const DevParams &p) {
   const int lane = threadIdx.x & 31;
   constexpr int K = kBuckets / 32;
-  float v[K];
-#pragma unroll
-  for (int k = 0; k < K; k++) v[k] = __uint_as_float(__ldcg(raw + lane * K + k));
-  float run = __int_as_float(0x7f800000);
-  float ex[K];
-#pragma unroll
+  const int j0 = lane * K;
+  unsigned int tot = 0x7f800000u;
   for (int k = 0; k < K; k++) {
-    ex[k] = run;
-    run = fminf(run, v[k]);
+    tot = min(tot, __ldcg(p.stv + j0 + k));
+    const unsigned long long x = __ldcg(p.stp + j0 + k);
+    if (x < s.bp[j0 + k]) atomicMin(s.bp + j0 + k, x);
   }
-  // exclusive scan of lane totals
-  float pre = run;
+  unsigned int pre = tot;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    float x = __shfl_up_sync(0xffffffffu, pre, o);
-    if (lane >= o) pre = fminf(pre, x);
+    const unsigned int x = __shfl_up_sync(0xffffffffu, pre, o);
+    if (lane >= o) pre = min(pre, x);
   }
-  float excl = __shfl_up_sync(0xffffffffu, pre, 1);
-  if (lane == 0) excl = __int_as_float(0x7f800000);
-#pragma unroll
-  for (int k = 0; k < K; k++) pm[lane * K + k] = fminf(excl, ex[k]);
+  unsigned int run = __shfl_up_sync(0xffffffffu, pre, 1);
+  if (lane == 0) run = 0x7f800000u;
+  for (int k = 0; k < K; k++) {
+    if (run < s.pm[j0 + k]) atomicMin(s.pm + j0 + k, run);
+    run = min(run, __ldcg(p.stv + j0 + k));
+  }
+  __threadfence_block();
   __syncwarp();
+}
+
+// T: exact canonical fp64 makespan (or a lower bound of it that is itself an
+// exact canonical makespan); eh: fp32 normalised energy (or a lower bound).
+__device__ __forceinline__ bool stair_dominated(const Stair &s, const DevParams &p, double T, float eh) {
+  const int j = bucket_of(T, p.bucket_base);
+  const unsigned int eb = __float_as_uint(eh);
+  if (eb > s.pm[j]) return true;
+  const unsigned long long pr = s.bp[j];
+  if (eb > (unsigned int)(pr >> 32)) {
+    const CandRec *c = (const CandRec *)p.cand + (unsigned int)pr;
+    return T >= __ldcg(&c->t);
+  }
+  return false;
 }
 
 // ---------------------------------------------------------- fp64 refine
@@ -188,9 +221,14 @@ __device__ __forceinline__ void warp_best(BestRec &b) {
 
 // Record a refined (fp64-exact) feasible configuration as a Pareto candidate
 // and tighten the staircases (sound: only verified points enter).
-__device__ __forceinline__ void emit_candidate(const DevParams &p, float *pm, u64 idx, double T, double E,
+__device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 idx, double T, double E,
                                                float t32, float e32) {
   const unsigned long long slot = atomicAdd(p.ctr + kCtrCand, 1ull);
+  const double g1 = 1.0 + (double)p.gamma;
+  const float val = __double2float_ru(__dmul_ru(__ddiv_ru(E, p.eseq), g1));
+  const unsigned int vb = __float_as_uint(val);
+  const int jb = bucket_of(T, p.bucket_base);
+  if (vb < __ldcg(p.stv + jb)) atomicMin(p.stv + jb, vb);
   if (slot < p.cand_cap) {
     CandRec *c = (CandRec *)p.cand + slot;
     c->idx = idx;
@@ -198,15 +236,143 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, float *pm, u6
     c->e = E;
     c->t32 = t32;
     c->e32 = e32;
+    __threadfence();  // the record is visible before its slot is published
+    const unsigned long long pr = ((unsigned long long)vb << 32) | slot;
+    if (pr < __ldcg(p.stp + jb)) {
+      atomicMin(p.stp + jb, pr);
+      atomicAdd(p.ctr + kCtrStairVer, 1ull);
+    }
+    atomicMin(s.bp + jb, pr);
   } else {
     atomicExch(p.ctr + kCtrOverflow, 1ull);
+    atomicAdd(p.ctr + kCtrStairVer, 1ull);
   }
-  const double g1 = 1.0 + (double)p.gamma;
-  const float key = __double2float_ru(__dmul_ru(__ddiv_ru(T, p.tseq), g1));
-  const float val = __double2float_ru(__dmul_ru(__ddiv_ru(E, p.eseq), g1));
-  const int jb = bucket_of(key, p.bucket_base);
-  atomicMin(p.stair + jb, __float_as_uint(val));
-  for (int i = jb + 1; i < kBuckets; i++) atomicMin((unsigned int *)pm + i, __float_as_uint(val));
+  const int hi = jb + 64 < kBuckets ? jb + 64 : kBuckets;
+  for (int i = jb + 1; i < hi; i++) atomicMin(s.pm + i, vb);
+}
+
+// ------------------------------------------------------------ DP walk (RGS state)
+struct LaneCfg {
+  int8_t a[kMaxN];
+  uint16_t st[kMaxN];   // st[i] = DP state after placing element i
+  uint32_t mask[kMaxG];
+  int8_t sz[kMaxG];
+  int k;
+  u64 v, Pn;            // level residue in [0, Pn), Pn = L^(#digits)
+  bool feasible;
+};
+
+__device__ __forceinline__ void cfg_feasibility(const Tables &tb, const DevParams &p, LaneCfg &c) {
+  bool ok = true;
+  for (int g = 0; g < c.k; g++) {
+    long long M = 0;
+    for (uint32_t mm = c.mask[g]; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
+    ok &= M <= (long long)p.mem_cap;
+  }
+  c.feasible = ok;
+}
+
+__device__ __forceinline__ int col_for(const DevParams &p, int j, int b, const int8_t *sz) {
+  if (j < b) {
+    if (p.capped) return sz[j] >= p.c ? -1 : sz[j];
+    return 1;
+  }
+  return b >= p.g ? -1 : 0;
+}
+
+__device__ __forceinline__ void place(LaneCfg &c, int i, int j) {
+  c.a[i] = (int8_t)j;
+  if (j == c.k) {
+    c.sz[c.k] = 0;
+    c.mask[c.k] = 0;
+    c.k++;
+  }
+  c.sz[j]++;
+  c.mask[j] |= 1u << i;
+}
+
+// index -> (RGS, residue) through the DP count table (R4 index order)
+static __device__ bool dev_unrank(const Tables &tb, const DevParams &p, u64 idx, LaneCfg &c) {
+  u64 r = idx;
+  int s = p.root;
+  c.k = 0;
+  place(c, 0, 0);
+  c.st[0] = (uint16_t)s;
+  for (int i = 1; i < p.n; i++) {
+    int chosen = -1;
+    for (int j = 0; j <= c.k; j++) {
+      const int col = col_for(p, j, c.k, c.sz);
+      if (col < 0) {
+        if (j == c.k) break;
+        continue;
+      }
+      const uint16_t s2 = tb.trans[s * p.tc + col];
+      if (s2 == kNoState) continue;
+      const u64 w = tb.W[s2];
+      if (r < w) {
+        chosen = j;
+        s = s2;
+        break;
+      }
+      r -= w;
+    }
+    if (chosen < 0) return false;
+    place(c, i, chosen);
+    c.st[i] = (uint16_t)s;
+  }
+  c.Pn = tb.W[c.st[p.n - 1]];
+  c.v = r;
+  cfg_feasibility(tb, p, c);
+  return true;
+}
+
+// next RGS in lexicographic order (valid + completable), digits reset by caller
+static __device__ bool dev_successor(const Tables &tb, const DevParams &p, LaneCfg &c) {
+  for (int i = p.n - 1; i >= 1; i--) {
+    const int j0 = c.a[i];
+    c.mask[j0] &= ~(1u << i);
+    if (--c.sz[j0] == 0) c.k--;
+    const int s = c.st[i - 1];
+    for (int j = j0 + 1; j <= c.k; j++) {
+      const int col = col_for(p, j, c.k, c.sz);
+      if (col < 0) {
+        if (j == c.k) break;
+        continue;
+      }
+      const uint16_t s2 = tb.trans[s * p.tc + col];
+      if (s2 == kNoState || tb.W[s2] == 0) continue;
+      place(c, i, j);
+      c.st[i] = s2;
+      for (int m = i + 1; m < p.n; m++) {  // greedy lexicographically-smallest completion
+        const int sm = c.st[m - 1];
+        for (int jj = 0; jj <= c.k; jj++) {
+          const int cl = col_for(p, jj, c.k, c.sz);
+          if (cl < 0) {
+            if (jj == c.k) break;
+            continue;
+          }
+          const uint16_t t2 = tb.trans[sm * p.tc + cl];
+          if (t2 == kNoState || tb.W[t2] == 0) continue;
+          place(c, m, jj);
+          c.st[m] = t2;
+          break;
+        }
+      }
+      return true;
+    }
+  }
+  return false;
+}
+
+__device__ __forceinline__ bool dev_advance(const Tables &tb, const DevParams &p, LaneCfg &c, u64 m) {
+  c.v += m;
+  while (c.v >= c.Pn) {
+    c.v -= c.Pn;
+    if (!dev_successor(tb, p, c)) return false;
+    c.Pn = tb.W[c.st[p.n - 1]];
+    cfg_feasibility(tb, p, c);
+  }
+  return true;
 }
 
 }  // namespace sched

@@ -387,11 +387,6 @@ double host_objective(double tseq, double eseq, double T, double E, int a, int b
 // ------------------------------------------------------------ staged tables
 static uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
 
-static uint32_t fbits(float f) {
-  uint32_t u;
-  std::memcpy(&u, &f, 4);
-  return u;
-}
 
 int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<unsigned char> *blob,
                 DevParams *dp) {
@@ -432,6 +427,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
     dp->delta[w] = (float)(4.0 * eta);
   }
   dp->gamma = (float)(2.0 * std::max(eT, eE) + 4.0 * u);
+  dp->tlb_scale = std::nextafter(tseq / (1.0 + 2.0 * eT), 0.0);
   // ---- tables ----
   uint32_t off = 0;
   auto take = [&](uint32_t bytes, uint32_t al) {
@@ -483,7 +479,12 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
               i == j ? 0.f : P.d[((size_t)(i * P.lp + q.lev[l]) * P.n + j) * P.lp + q.lev[m]];
         }
   }
-  dp->bucket_base = fbits(tlow * 0.5f) >> kBucketShift;
+  {
+    const double tl = (double)tlow * 0.5 * tseq;
+    uint64_t b;
+    std::memcpy(&b, &tl, 8);
+    dp->bucket_base = (uint32_t)(b >> kBucketShift);
+  }
   std::memcpy(B + dp->off_W, sp.W.data(), 8 * sp.W.size());
   std::memcpy(B + dp->off_trans, sp.trans.data(), 2 * sp.trans.size());
   // ---- work split: chunks c with c % count == rank ----
@@ -503,6 +504,12 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   }
   dp->n_units = dp->n_owned << (dp->chunk_log2 - dp->unit_log2);
   dp->cand_cap = q.cand_cap;
+  {  // interleave lanes when partitions hold enough level vectors to keep lanes together
+    double per = 1.0;
+    const int nd = q.scope == SCHED_PER_CLIENT ? n : std::min(q.g, n);
+    for (int k = 0; k < nd; k++) per *= L;
+    dp->lane_strided = per >= 64.0;
+  }
   return SCHED_OK;
 }
 

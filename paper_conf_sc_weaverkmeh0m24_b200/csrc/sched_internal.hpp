@@ -16,8 +16,8 @@ constexpr int kMaxN = SCHED_MAX_WORKFLOWS;      // 32
 constexpr int kMaxG = SCHED_MAX_GPUS;           // 16
 constexpr int kMaxL = SCHED_MAX_SEARCH_LEVELS;  // 8
 constexpr int kMaxW = SCHED_MAX_WEIGHTS;        // 8
-constexpr int kBuckets = 256;                   // Pareto staircase buckets (per warp)
-constexpr int kBucketShift = 18;                // 32 buckets per binade of T/T_seq
+constexpr int kBuckets = 2048;                  // Pareto staircase buckets (per CTA)
+constexpr int kBucketShift = 45;                // of the fp64 bits of T: 128 buckets per binade
 constexpr uint16_t kNoState = 0xFFFF;
 constexpr int kUnitLog2 = 11;                   // generic kernel: 2048 configs per warp unit
 
@@ -64,15 +64,18 @@ struct DevParams {
   int wa[kMaxW], wb[kMaxW];
   float delta[kMaxW];       // fp32 screen margin per weight
   float gamma;              // Pareto "surely dominated" margin
+  int ws_perm[kMaxW];       // tile kernel: compile-time weight slot -> query weight index
+  double tlb_scale;         // T_seq / (1 + 2 eps_T) rounded down: T64 >= T32hat * tlb_scale
   float phat;               // P_s * T_seq / E_seq
   double ps, tseq, eseq;
   int mem_cap, want_pareto, root, nstates;
-  uint32_t bucket_base;     // (bits(T_lower) >> kBucketShift)
+  uint32_t bucket_base;     // (bits64(T_lower) >> kBucketShift)
   // work split
   uint64_t lo, hi;          // window
   uint64_t first_chunk;     // first owned chunk id
   uint64_t n_owned;         // owned chunks intersecting [lo, hi)
   int shard_count, chunk_log2, unit_log2;
+  int lane_strided;         // generic kernel: lanes interleave indices (1) or take contiguous runs (0)
   uint64_t n_units;
   // staged blob offsets (bytes from blob start) and size
   uint32_t off_th, off_u, off_bw, off_dh, off_traw, off_praw, off_mem, off_d, off_W, off_trans;
@@ -81,7 +84,8 @@ struct DevParams {
   const unsigned char *blob;   // staged tables (device)
   unsigned long long *ctr;     // counters (see kCtr*)
   unsigned int *thr;           // [kMaxW] global fp32 proxy threshold bits (min)
-  unsigned int *stair;         // [kBuckets] raw staircase (float bits, min)
+  unsigned int *stv;           // [kBuckets] min val of verified points per bucket
+  unsigned long long *stp;     // [kBuckets] min (val << 32 | candidate slot) per bucket
   unsigned char *slots;        // [grid][W] BestRec
   unsigned char *cand;         // [cand_cap] CandRec
   uint32_t cand_cap;
@@ -97,6 +101,8 @@ enum {
   kCtrOverflow = 5,  // candidate overflow flag
   kCtrSurv = 6,      // finalize: Pareto survivors
   kCtrFront = 7,     // finalize: front size
+  kCtrStairVer = 8,  // staircase version (bumped per insertion)
+  kCtrPass = 9,      // search passes run
   kCtrN = 16
 };
 

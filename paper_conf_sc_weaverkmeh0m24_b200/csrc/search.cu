@@ -18,133 +18,9 @@
 #include <cstring>
 
 #include "device_common.cuh"
-#include "search_tile.cuh"
+#include "tile_registry.hpp"
 
 namespace sched {
-
-// ------------------------------------------------------------ lane state
-struct LaneCfg {
-  int8_t a[kMaxN];
-  uint16_t st[kMaxN];   // st[i] = DP state after placing element i
-  uint32_t mask[kMaxG];
-  int8_t sz[kMaxG];
-  int k;
-  u64 v, Pn;            // level residue in [0, Pn), Pn = L^(#digits)
-  bool feasible;
-};
-
-__device__ __forceinline__ void cfg_feasibility(const Tables &tb, const DevParams &p, LaneCfg &c) {
-  bool ok = true;
-  for (int g = 0; g < c.k; g++) {
-    long long M = 0;
-    for (uint32_t mm = c.mask[g]; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
-    ok &= M <= (long long)p.mem_cap;
-  }
-  c.feasible = ok;
-}
-
-__device__ __forceinline__ int col_for(const DevParams &p, int j, int b, const int8_t *sz) {
-  if (j < b) {
-    if (p.capped) return sz[j] >= p.c ? -1 : sz[j];
-    return 1;
-  }
-  return b >= p.g ? -1 : 0;
-}
-
-__device__ __forceinline__ void place(LaneCfg &c, int i, int j) {
-  c.a[i] = (int8_t)j;
-  if (j == c.k) {
-    c.sz[c.k] = 0;
-    c.mask[c.k] = 0;
-    c.k++;
-  }
-  c.sz[j]++;
-  c.mask[j] |= 1u << i;
-}
-
-// index -> (RGS, residue) through the DP count table (R4 index order)
-__device__ bool dev_unrank(const Tables &tb, const DevParams &p, u64 idx, LaneCfg &c) {
-  u64 r = idx;
-  int s = p.root;
-  c.k = 0;
-  place(c, 0, 0);
-  c.st[0] = (uint16_t)s;
-  for (int i = 1; i < p.n; i++) {
-    int chosen = -1;
-    for (int j = 0; j <= c.k; j++) {
-      const int col = col_for(p, j, c.k, c.sz);
-      if (col < 0) {
-        if (j == c.k) break;
-        continue;
-      }
-      const uint16_t s2 = tb.trans[s * p.tc + col];
-      if (s2 == kNoState) continue;
-      const u64 w = tb.W[s2];
-      if (r < w) {
-        chosen = j;
-        s = s2;
-        break;
-      }
-      r -= w;
-    }
-    if (chosen < 0) return false;
-    place(c, i, chosen);
-    c.st[i] = (uint16_t)s;
-  }
-  c.Pn = tb.W[c.st[p.n - 1]];
-  c.v = r;
-  cfg_feasibility(tb, p, c);
-  return true;
-}
-
-// next RGS in lexicographic order (valid + completable), digits reset by caller
-__device__ bool dev_successor(const Tables &tb, const DevParams &p, LaneCfg &c) {
-  for (int i = p.n - 1; i >= 1; i--) {
-    const int j0 = c.a[i];
-    c.mask[j0] &= ~(1u << i);
-    if (--c.sz[j0] == 0) c.k--;
-    const int s = c.st[i - 1];
-    for (int j = j0 + 1; j <= c.k; j++) {
-      const int col = col_for(p, j, c.k, c.sz);
-      if (col < 0) {
-        if (j == c.k) break;
-        continue;
-      }
-      const uint16_t s2 = tb.trans[s * p.tc + col];
-      if (s2 == kNoState || tb.W[s2] == 0) continue;
-      place(c, i, j);
-      c.st[i] = s2;
-      for (int m = i + 1; m < p.n; m++) {  // greedy lexicographically-smallest completion
-        const int sm = c.st[m - 1];
-        for (int jj = 0; jj <= c.k; jj++) {
-          const int cl = col_for(p, jj, c.k, c.sz);
-          if (cl < 0) {
-            if (jj == c.k) break;
-            continue;
-          }
-          const uint16_t t2 = tb.trans[sm * p.tc + cl];
-          if (t2 == kNoState || tb.W[t2] == 0) continue;
-          place(c, m, jj);
-          c.st[m] = t2;
-          break;
-        }
-      }
-      return true;
-    }
-  }
-  return false;
-}
-
-__device__ __forceinline__ bool dev_advance(const Tables &tb, const DevParams &p, LaneCfg &c, u64 m) {
-  c.v += m;
-  while (c.v >= c.Pn) {
-    c.v -= c.Pn;
-    if (!dev_successor(tb, p, c)) return false;
-    c.Pn = tb.W[c.st[p.n - 1]];
-    cfg_feasibility(tb, p, c);
-  }
-  return true;
-}
 
 __device__ __forceinline__ void decode_levels(const DevParams &p, const LaneCfg &c, int *lam) {
   const int nd = p.scope == SCHED_PER_CLIENT ? p.n : c.k;
@@ -200,8 +76,12 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
   stage_blob(sm, p);
   const Tables tb = tables_at(sm, p);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  float *pm = (float *)(sm + ((p.blob_bytes + 15) & ~15u)) + warp * kBuckets;
-  BestRec *red = (BestRec *)((float *)(sm + ((p.blob_bytes + 15) & ~15u)) + kWarps * kBuckets);
+  unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
+  Stair stair{(unsigned int *)(after + 8 * kBuckets), (unsigned long long *)after};
+  BestRec *red = (BestRec *)(after + 12 * kBuckets);
+  stair_init(stair);
+  __syncthreads();
+  u64 stair_ver = 0;
 
   float thr[kMaxW];
   BestRec lb[kMaxW];
@@ -230,10 +110,20 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
 #pragma unroll
     for (int w = 0; w < kMaxW; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
-    if (p.want_pareto) refresh_stair(pm, p.stair);
+    if (p.want_pareto) {
+      const u64 v = __ldcg(p.ctr + kCtrStairVer);
+      if (v != stair_ver) {
+        stair_ver = v;
+        stair_merge(stair, p);
+      }
+    }
 
-    u64 idx = s + lane;
-    if (idx < e && dev_unrank(tb, p, idx, c)) {
+    // lanes interleave (idx = s + lane + 32 j) or take contiguous runs
+    const u64 run = p.lane_strided ? 0 : (e - s + 31) / 32;
+    u64 idx = p.lane_strided ? s + lane : s + lane * run;
+    const u64 lend = p.lane_strided ? e : (idx + run < e ? idx + run : e);
+    const u64 step = p.lane_strided ? 32 : 1;
+    if (idx < lend && dev_unrank(tb, p, idx, c)) {
       for (;;) {
         ncfg++;
         if (c.feasible) {
@@ -255,7 +145,9 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
             }
           }
           bool par = false;
-          if (p.want_pareto) par = !(E > pm[bucket_of(T, p.bucket_base)]);
+          if (p.want_pareto) {  // certified lower bound of the exact T (sound screen)
+            par = !stair_dominated(stair, p, __dmul_rd((double)T, p.tlb_scale), E);
+          }
           if (need || par) {
             nref++;
             double T64, E64;
@@ -275,12 +167,13 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
                 }
               }
             }
-            if (par) emit_candidate(p, pm, idx, T64, E64, T, E);
+            if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))))
+              emit_candidate(p, stair, idx, T64, E64, T, E);
           }
         }
-        idx += 32;
-        if (idx >= e) break;
-        if (!dev_advance(tb, p, c, 32)) break;
+        idx += step;
+        if (idx >= lend) break;
+        if (!dev_advance(tb, p, c, step)) break;
       }
     }
     __syncwarp();
@@ -328,11 +221,53 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
 }
 
 // ------------------------------------------------------------ init / finalize
-__global__ void k_init(const DevParams p) {
+__global__ void k_init(const DevParams p, int keep_stair) {
   const int t = threadIdx.x;
-  if (t < kCtrN) p.ctr[t] = 0ull;
+  if (t < kCtrN && !(keep_stair && (t == kCtrStairVer || t == kCtrPass))) p.ctr[t] = 0ull;
+  if (keep_stair) return;
   if (t < kMaxW) p.thr[t] = 0x7f800000u;
-  for (int i = t; i < kBuckets; i += blockDim.x) p.stair[i] = 0x7f800000u;
+  for (int i = t; i < kBuckets; i += blockDim.x) {
+    p.stv[i] = 0x7f800000u;
+    p.stp[i] = ~0ull;
+  }
+}
+
+// Before a seeded re-run: keep only the candidate records the same-bucket
+// staircase references (compacted to slots 0..m-1, ids rewritten), so the
+// re-run's candidate buffer starts with them.  One block of 1024 threads.
+__global__ void __launch_bounds__(1024) k_reseed(const DevParams p, CandRec *tmp) {
+  __shared__ unsigned int cnt[1024];
+  constexpr int K = kBuckets / 1024;
+  const int t = threadIdx.x;
+  unsigned int mine = 0;
+  for (int k = 0; k < K; k++) {
+    const int j = t * K + k;
+    const unsigned long long x = p.stp[j];
+    if (x != ~0ull) {
+      tmp[j] = ((const CandRec *)p.cand)[(unsigned int)x];
+      mine++;
+    }
+  }
+  cnt[t] = mine;
+  __syncthreads();
+  for (int o = 1; o < 1024; o <<= 1) {  // inclusive scan
+    const unsigned int v = t >= o ? cnt[t - o] : 0u;
+    __syncthreads();
+    cnt[t] += v;
+    __syncthreads();
+  }
+  unsigned int slot = cnt[t] - mine;
+  for (int k = 0; k < K; k++) {
+    const int j = t * K + k;
+    const unsigned long long x = p.stp[j];
+    if (x != ~0ull) {
+      ((CandRec *)p.cand)[slot] = tmp[j];
+      p.stp[j] = (x & 0xffffffff00000000ull) | slot;
+      slot++;
+    }
+  }
+  __threadfence();
+  if (t == 1023) p.ctr[kCtrCand] = cnt[1023];
 }
 
 // best per weight over the per-CTA slots -> out[0 .. W)
@@ -360,14 +295,16 @@ __global__ void k_best_final(const DevParams p, int nslots) {
 // Pareto finalize, stage 1: drop candidates surely (strictly) dominated by a
 // verified point of the final global staircase; compact survivors.
 __global__ void k_pareto_prefilter(const DevParams p, int ncand, unsigned int *surv) {
-  __shared__ float pm[kBuckets];
-  if (threadIdx.x < 32) refresh_stair(pm, p.stair);
+  __shared__ unsigned int s_pm[kBuckets];
+  __shared__ unsigned long long s_bp[kBuckets];
+  Stair stair{s_pm, s_bp};
+  stair_init(stair);
+  __syncthreads();
+  if (threadIdx.x < 32) stair_merge(stair, p);
   __syncthreads();
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
     const CandRec c = ((const CandRec *)p.cand)[i];
-    const float tl = __double2float_rd(__ddiv_rd(c.t, p.tseq));
-    const float el = __double2float_rd(__ddiv_rd(c.e, p.eseq));
-    const bool dom = el > pm[bucket_of(tl, p.bucket_base)];
+    const bool dom = stair_dominated(stair, p, c.t, __double2float_rd(__ddiv_rd(c.e, p.eseq)));
     if (!dom) {
       const unsigned int k = (unsigned int)atomicAdd(p.ctr + kCtrSurv, 1ull);
       surv[k] = (unsigned int)i;
@@ -430,7 +367,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stair, blob, slots, cand, surv, keep, out, total;
+  size_t ctr, thr, stv, stp, blob, slots, cand, surv, keep, out, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -444,7 +381,8 @@ WsLayout layout(const DevParams &dp) {
   };
   L.ctr = take(8 * kCtrN);
   L.thr = take(4 * kMaxW);
-  L.stair = take(4 * kBuckets);
+  L.stv = take(4 * kBuckets);
+  L.stp = take(8 * kBuckets);
   L.blob = take(dp.blob_bytes);
   L.slots = take(sizeof(BestRec) * kMaxW * (size_t)kMaxGrid);
   L.cand = take(sizeof(CandRec) * (size_t)dp.cand_cap);
@@ -487,7 +425,8 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.blob = ws + L.blob;
   dp.ctr = (unsigned long long *)(ws + L.ctr);
   dp.thr = (unsigned int *)(ws + L.thr);
-  dp.stair = (unsigned int *)(ws + L.stair);
+  dp.stv = (unsigned int *)(ws + L.stv);
+  dp.stp = (unsigned long long *)(ws + L.stp);
   dp.slots = ws + L.slots;
   dp.cand = ws + L.cand;
   dp.out = ws + L.out;
@@ -500,35 +439,45 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   CK(cudaEventCreate(&e1));
   CK(cudaEventCreate(&e2));
   CK(cudaEventRecord(e0, st));
-  k_init<<<1, 256, 0, st>>>(dp);
-  CK(cudaGetLastError());
-
   int grid = 0, path = 0;
-  TileLaunch tl;
-  if (tile_eligible(dp, &tl)) {
-    path = 1;
-    CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid));
-  } else {
-    const size_t smem = ((dp.blob_bytes + 15) & ~15u) + sizeof(float) * kWarps * kBuckets +
-                        sizeof(BestRec) * kWarps * kMaxW;
-    CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    int occ = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_generic, kThreads, smem));
-    if (occ < 1) return SCHED_E_TOO_LARGE;
-    grid = std::min(kMaxGrid, nsm * occ);
-    CK(cudaEventRecord(e1, st));
-    k_generic<<<grid, kThreads, smem, st>>>(dp);
-    CK(cudaGetLastError());
-    CK(cudaEventRecord(e2, st));
-  }
-  // finalize
-  if (dp.nw > 0) {
-    k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid);
-    CK(cudaGetLastError());
-  }
+  float search_ms = 0.f;
   uint64_t ctr[kCtrN];
-  CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
-  CK(cudaStreamSynchronize(st));
+  // pass 0 from an empty staircase; on candidate-buffer overflow, pass 1
+  // re-runs seeded with pass 0's final staircase and thresholds (sound).
+  for (int pass = 0; pass < 2; pass++) {
+    k_init<<<1, 256, 0, st>>>(dp, pass > 0);
+    CK(cudaGetLastError());
+    if (pass > 0 && dp.want_pareto) {
+      k_reseed<<<1, 1024, 0, st>>>(dp, (CandRec *)dp.out);
+      CK(cudaGetLastError());
+    }
+    TileLaunch tl;
+    if (tile_eligible(dp, &tl)) {
+      path = 1;
+      CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid));
+    } else {
+      const size_t smem = ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(BestRec) * kWarps * kMaxW;
+      CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      int occ = 0;
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_generic, kThreads, smem));
+      if (occ < 1) return SCHED_E_TOO_LARGE;
+      grid = std::min(kMaxGrid, nsm * occ);
+      CK(cudaEventRecord(e1, st));
+      k_generic<<<grid, kThreads, smem, st>>>(dp);
+      CK(cudaGetLastError());
+      CK(cudaEventRecord(e2, st));
+    }
+    if (dp.nw > 0) {
+      k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid);
+      CK(cudaGetLastError());
+    }
+    CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, e1, e2));
+    search_ms += ms;
+    if (!ctr[kCtrOverflow]) break;
+  }
   int ncand = (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap);
   if (dp.want_pareto && ncand > 0) {
     unsigned int *surv = (unsigned int *)(ws + L.surv), *keep = (unsigned int *)(ws + L.keep);
@@ -551,9 +500,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
                        cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
   }
-  float ms = 0.f;
-  CK(cudaEventElapsedTime(&ms, e1, e2));
-  info->search_ms = ms;
+  info->search_ms = search_ms;
   info->grid = grid;
   info->path = path;
   for (int k = 0; k < kCtrN; k++) ctr_out[k] = ctr[k];

@@ -1,0 +1,78 @@
+// tile_host.cu -- weight-set matching and launch of the PER_GPU tile kernel.
+#include "search_tile.cuh"
+
+namespace sched {
+
+template <class WS>
+static bool ws_match(const DevParams &dp, int *perm) {
+  if (dp.nw != WS::N) return false;
+  bool used[kMaxW] = {false};
+  for (int s = 0; s < WS::N; s++) {
+    int found = -1;
+    for (int w = 0; w < dp.nw; w++)
+      if (!used[w] && dp.wa[w] == WS::A(s) && dp.wb[w] == WS::B(s)) {
+        found = w;
+        break;
+      }
+    if (found < 0) return false;
+    used[found] = true;
+    perm[s] = found;
+  }
+  return true;
+}
+
+template <int L>
+static const void *tile_pick_ws(DevParams *dp) {
+  int perm[kMaxW];
+#define TRY(WS)                                                 \
+  if (ws_match<WS>(*dp, perm) && (WS::N > 0 || dp->want_pareto)) { \
+    for (int s = 0; s < WS::N; s++) dp->ws_perm[s] = perm[s];     \
+    return tile_fn<L, WS>();                                    \
+  }
+  TRY(WS_P)
+  TRY(WS_11)
+  TRY(WS_10)
+  TRY(WS_01)
+  TRY(WS_11_21)
+#undef TRY
+  return nullptr;
+}
+
+size_t tile_smem_bytes(const DevParams &dp) {
+  return ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(WarpPart) * kTileWarps +
+         sizeof(BestRec) * kTileWarps * kMaxW;
+}
+
+bool tile_eligible(DevParams &dp, TileLaunch *tl) {
+  if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4) return false;
+  const void *fn = tile_pick_ws<4>(&dp);
+  if (!fn) return false;
+  tl->fn = fn;
+  tl->smem = tile_smem_bytes(dp);
+  return true;
+}
+
+cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                        cudaEvent_t e2, int *grid) {
+  cudaError_t err = cudaFuncSetAttribute(tl.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tl.smem);
+  if (err != cudaSuccess) return err;
+  int occ = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kTileThreads, tl.smem);
+  if (err != cudaSuccess) return err;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  *grid = std::min(4096, nsm * occ);
+  // unit size: ~16 units per warp over the search, 2^12 .. 2^chunk_log2 configs
+  const uint64_t range = dp.n_owned << dp.chunk_log2;
+  const uint64_t warps = (uint64_t)(*grid) * kTileWarps;
+  int ul = 12;
+  while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 16) ul++;
+  dp.unit_log2 = ul;
+  dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+  void *args[] = {(void *)&dp};
+  cudaEventRecord(e1, st);
+  err = cudaLaunchKernel(tl.fn, *grid, kTileThreads, args, tl.smem, st);
+  cudaEventRecord(e2, st);
+  return err;
+}
+
+}  // namespace sched

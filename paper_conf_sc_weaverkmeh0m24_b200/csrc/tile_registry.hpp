@@ -1,0 +1,35 @@
+// tile_registry.hpp -- host-side selection of the PER_GPU tile kernel.
+// The kernels are instantiated in tile_*.cu (one weight set per translation
+// unit, compiled in parallel); search.cu only sees these declarations.
+#pragma once
+#include <algorithm>
+#include <cuda_runtime.h>
+
+#include "sched_internal.hpp"
+
+namespace sched {
+
+struct WS_P;
+struct WS_11;
+struct WS_10;
+struct WS_01;
+struct WS_11_21;
+
+template <int L, class WS>
+const void *tile_fn();
+
+struct TileLaunch {
+  const void *fn;
+  size_t smem;
+};
+
+constexpr int kTileThreads = 256;
+constexpr int kTileWarps = kTileThreads / 32;
+constexpr int kTileMaxL = 4;
+constexpr int kTileMaxG = 8;
+size_t tile_smem_bytes(const DevParams &dp);
+bool tile_eligible(DevParams &dp, TileLaunch *tl);
+cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                        cudaEvent_t e2, int *grid);
+
+}  // namespace sched
