@@ -126,6 +126,10 @@ typedef struct {
   float total_ms;               /* device time of the whole call on the stream */
   int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile kernel, 2 partition DFS kernel */
   int32_t grid_ctas;            /* persistent CTAs launched by the search kernel */
+  int32_t kernel_launches;      /* kernels this call launched (init, search pass(es), finalize) */
+  int32_t passes;               /* search passes (2 = re-run after candidate overflow) */
+  uint64_t h2d_bytes;           /* host->device bytes this call copied (staged tables) */
+  uint64_t d2h_bytes;           /* device->host bytes this call copied (counters, picks) */
 } sched_stats;
 
 typedef struct sched_handle sched_handle;

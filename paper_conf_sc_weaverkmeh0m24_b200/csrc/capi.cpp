@@ -204,9 +204,11 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
   cudaEvent_t t0, t1;
   if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess) return SCHED_E_CUDA;
   cudaEventRecord(t0, (cudaStream_t)stream);
+  uint64_t h2d = 0;
   if (h->staged_ws != ws || h->staged_blob != blob) {
     st = do_stage(h, dp, blob, ws, stream);
     if (st) return st;
+    h2d = blob.size();
   }
   LaunchInfo info;
   std::vector<BestRec> bres;
@@ -257,6 +259,10 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
     stats->total_ms = total_ms;
     stats->kernel_path = info.path;
     stats->grid_ctas = info.grid;
+    stats->kernel_launches = info.launches;
+    stats->passes = info.passes;
+    stats->h2d_bytes = h2d;
+    stats->d2h_bytes = info.d2h_bytes;
   }
   if (st) return st;
   if (ctr[kCtrFeasible] == 0) return SCHED_E_INFEASIBLE;

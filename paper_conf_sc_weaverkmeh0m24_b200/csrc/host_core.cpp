@@ -428,6 +428,11 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   }
   dp->gamma = (float)(2.0 * std::max(eT, eE) + 4.0 * u);
   dp->tlb_scale = std::nextafter(tseq / (1.0 + 2.0 * eT), 0.0);
+  {
+    float f = (float)dp->tlb_scale;
+    if ((double)f > dp->tlb_scale) f = std::nextafter(f, 0.f);
+    dp->tlb_scale_f = f;
+  }
   // ---- tables ----
   uint32_t off = 0;
   auto take = [&](uint32_t bytes, uint32_t al) {
@@ -503,6 +508,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
     dp->n_owned = f > c1 ? 0 : (c1 - f) / R64 + 1;
   }
   dp->n_units = dp->n_owned << (dp->chunk_log2 - dp->unit_log2);
+  dp->unit_stride = 1;
   dp->cand_cap = q.cand_cap;
   {  // interleave lanes when partitions hold enough level vectors to keep lanes together
     double per = 1.0;

@@ -66,6 +66,7 @@ struct DevParams {
   float gamma;              // Pareto "surely dominated" margin
   int ws_perm[kMaxW];       // tile kernel: compile-time weight slot -> query weight index
   double tlb_scale;         // T_seq / (1 + 2 eps_T) rounded down: T64 >= T32hat * tlb_scale
+  float tlb_scale_f;        // the same, as a float rounded down
   float phat;               // P_s * T_seq / E_seq
   double ps, tseq, eseq;
   int mem_cap, want_pareto, root, nstates;
@@ -77,6 +78,7 @@ struct DevParams {
   int shard_count, chunk_log2, unit_log2;
   int lane_strided;         // generic kernel: lanes interleave indices (1) or take contiguous runs (0)
   uint64_t n_units;
+  uint64_t unit_stride;      // unit u covers global unit u * unit_stride (seed pass samples)
   // staged blob offsets (bytes from blob start) and size
   uint32_t off_th, off_u, off_bw, off_dh, off_traw, off_praw, off_mem, off_d, off_W, off_trans;
   uint32_t blob_bytes;
@@ -139,8 +141,9 @@ int merge_picks(int n_ranks, int nw, const sched_pick *rank_best, const sched_pi
 
 // ---- device launchers (search.cu) ----
 struct LaunchInfo {
-  int path, grid;
+  int path, grid, launches, passes;
   float search_ms;
+  uint64_t d2h_bytes;
 };
 size_t workspace_bytes(const DevParams &dp, int max_grid);
 int stage_tables(const DevParams &dp, const std::vector<unsigned char> &blob, void *d_ws, void *host_pinned,

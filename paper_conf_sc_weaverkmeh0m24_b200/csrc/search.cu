@@ -100,8 +100,9 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
     if (lane == 0) unit = atomicAdd(p.ctr + kCtrUnit, 1ull);
     unit = __shfl_sync(0xffffffffu, unit, 0);
     if (unit >= p.n_units) break;
-    const u64 ch = p.first_chunk + (unit >> (cl - ul)) * (u64)p.shard_count;
-    u64 s = (ch << cl) + ((unit & ((1ull << (cl - ul)) - 1)) << ul);
+    const u64 ue = unit * p.unit_stride;
+    const u64 ch = p.first_chunk + (ue >> (cl - ul)) * (u64)p.shard_count;
+    u64 s = (ch << cl) + ((ue & ((1ull << (cl - ul)) - 1)) << ul);
     u64 e = s + (1ull << ul);
     s = s > p.lo ? s : p.lo;
     e = e < p.hi ? e : p.hi;
@@ -221,10 +222,15 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
 }
 
 // ------------------------------------------------------------ init / finalize
-__global__ void k_init(const DevParams p, int keep_stair) {
+// keep = 0: fresh search; 1: seeded re-run after overflow (keep staircase +
+// thresholds, drop candidates); 2: after the seed pass (keep staircase,
+// thresholds and the seed pass's in-range candidates).
+__global__ void k_init(const DevParams p, int keep) {
   const int t = threadIdx.x;
-  if (t < kCtrN && !(keep_stair && (t == kCtrStairVer || t == kCtrPass))) p.ctr[t] = 0ull;
-  if (keep_stair) return;
+  const bool kept = keep && (t == kCtrStairVer || t == kCtrPass ||
+                             (keep == 2 && (t == kCtrCand || t == kCtrOverflow)));
+  if (t < kCtrN && !kept) p.ctr[t] = 0ull;
+  if (keep) return;
   if (t < kMaxW) p.thr[t] = 0x7f800000u;
   for (int i = t; i < kBuckets; i += blockDim.x) {
     p.stv[i] = 0x7f800000u;
@@ -439,22 +445,39 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   CK(cudaEventCreate(&e1));
   CK(cudaEventCreate(&e2));
   CK(cudaEventRecord(e0, st));
-  int grid = 0, path = 0;
+  int grid = 0, path = 0, launches = 0, passes = 0;
+  uint64_t d2h = 0;
   float search_ms = 0.f;
   uint64_t ctr[kCtrN];
   // pass 0 from an empty staircase; on candidate-buffer overflow, pass 1
   // re-runs seeded with pass 0's final staircase and thresholds (sound).
-  for (int pass = 0; pass < 2; pass++) {
-    k_init<<<1, 256, 0, st>>>(dp, pass > 0);
+  // pass 0: seed pass over a sample of in-range units (2^12 configs each,
+  // spread over the shard) that fills the staircase and thresholds; pass 1:
+  // the full search; pass 2 only after a candidate-buffer overflow.
+  const DevParams dp_full = dp;
+  const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
+                    (dp.n_owned << (dp.chunk_log2 - 12)) >= (uint64_t)nsm * 64 * 16;
+  for (int pass = seed ? 0 : 1; pass < 3; pass++) {
+    dp = dp_full;
+    if (pass == 0) {
+      const uint64_t u12 = dp.n_owned << (dp.chunk_log2 - 12);
+      dp.unit_log2 = 12;
+      dp.n_units = (uint64_t)nsm * 64;
+      dp.unit_stride = u12 / dp.n_units;
+    }
+    passes++;
+    k_init<<<1, 256, 0, st>>>(dp, pass == 0 ? 0 : (pass == 1 ? (seed ? 2 : 0) : 1));
     CK(cudaGetLastError());
-    if (pass > 0 && dp.want_pareto) {
+    launches++;
+    if (pass == 2 && dp.want_pareto) {
       k_reseed<<<1, 1024, 0, st>>>(dp, (CandRec *)dp.out);
       CK(cudaGetLastError());
+      launches++;
     }
     TileLaunch tl;
     if (tile_eligible(dp, &tl)) {
       path = 1;
-      CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid));
+      CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
     } else {
       const size_t smem = ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(BestRec) * kWarps * kMaxW;
       CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
@@ -467,16 +490,19 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       CK(cudaGetLastError());
       CK(cudaEventRecord(e2, st));
     }
+    launches++;
     if (dp.nw > 0) {
       k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid);
       CK(cudaGetLastError());
+      launches++;
     }
     CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
+    d2h += sizeof ctr;
     CK(cudaStreamSynchronize(st));
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, e1, e2));
     search_ms += ms;
-    if (!ctr[kCtrOverflow]) break;
+    if (pass >= 1 && !ctr[kCtrOverflow]) break;
   }
   int ncand = (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap);
   if (dp.want_pareto && ncand > 0) {
@@ -488,21 +514,27 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     k_pareto_order<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, surv, keep,
                                                                                         kFrontCap);
     CK(cudaGetLastError());
+    launches += 3;
   }
   CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
   best->resize(kMaxW);
   CK(cudaMemcpyAsync(best->data(), dp.out, sizeof(BestRec) * kMaxW, cudaMemcpyDeviceToHost, st));
+  d2h += sizeof ctr + sizeof(BestRec) * kMaxW;
   CK(cudaStreamSynchronize(st));
   const uint64_t nfront = dp.want_pareto && ncand > 0 ? ctr[kCtrFront] : 0;
   pareto->resize(std::min<uint64_t>(nfront, kFrontCap));
   if (!pareto->empty()) {
     CK(cudaMemcpyAsync(pareto->data(), dp.out + sizeof(BestRec) * kMaxW, sizeof(CandRec) * pareto->size(),
                        cudaMemcpyDeviceToHost, st));
+    d2h += sizeof(CandRec) * pareto->size();
     CK(cudaStreamSynchronize(st));
   }
   info->search_ms = search_ms;
   info->grid = grid;
   info->path = path;
+  info->launches = launches;
+  info->passes = passes;
+  info->d2h_bytes = d2h;
   for (int k = 0; k < kCtrN; k++) ctr_out[k] = ctr[k];
   ctr_out[kCtrFront] = nfront;
   cudaEventDestroy(e0);

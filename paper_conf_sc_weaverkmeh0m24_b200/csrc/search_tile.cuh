@@ -86,8 +86,9 @@ struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
 struct WarpPart {
   LaneCfg cfg;
   u64 base;
-  float gt[kTileMaxG * kTileMaxL], ge[kTileMaxG * kTileMaxL];
-  double g64[kTileMaxG * kTileMaxL];
+  float gt[kTileMaxG * 4], ge[kTileMaxG * 4];
+  double g64[kTileMaxG * 4];
+  float2 lp[64];  // loop-prefix (max T, sum E) over groups 0..k-6, one entry per digit string
 };
 
 // fp32 + exact fp64 makespan of group `m` with every member at level mu
@@ -129,41 +130,53 @@ __device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p,
 }
 
 template <class WS>
-struct LaneAcc {
-  float thr[WS::N > 0 ? WS::N : 1];
-  BestRec lb[WS::N > 0 ? WS::N : 1];
-  u64 nref;
+struct Thr {
+  float v[WS::N > 0 ? WS::N : 1];
 };
 
-// One configuration (digits dig[0..K-1], exact T64 and fp32 T/E): per-weight
-// screen, Pareto screen, fp64 refine, record.  Slow path.
-template <int L, class WS, int K>
-__device__ __noinline__ void check_config(const Tables &tb, const DevParams &p, const Stair &stair,
-                                             const WarpPart &wp, LaneAcc<WS> &acc, u64 idx,
-                                             const int *dig, float T, float E, double T64) {
+// quick Pareto screen from fp32 values: tlb = certified lower bound of the
+// exact makespan T (unnormalised, float, rounded down), eh = fp32 E/E_seq.
+// Buckets of a float coincide with buckets of the same value as a double.
+__device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParams &p, float tlb, float eh) {
+  const int b = (int)((__float_as_uint(tlb) >> 16) + (896u << 7)) - (int)p.bucket_base;
+  const int j = b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
+  const unsigned int eb = __float_as_uint(eh);
+  if (eb > s.pm[j]) return true;
+  const unsigned long long pr = s.bp[j];
+  if (eb > (unsigned int)(pr >> 32)) {
+    const CandRec *c = (const CandRec *)p.cand + (unsigned int)pr;
+    return (double)tlb >= __ldcg(&c->t);
+  }
+  return false;
+}
+
+// One configuration of the current partition (level digits dig[0..k-1],
+// exact T64, fp32 T/E): per-weight screen, Pareto screen, fp64 refine,
+// record.  Out of line (slow path).  Returns 1 if it issued a refine.
+template <class WS>
+__device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, const Stair &stair,
+                                         const WarpPart &wp, const Thr<WS> thr, BestRec *lb, u64 idx,
+                                         const int *dig, float T, float E, double T64) {
   unsigned need = 0;
   if constexpr (WS::N > 0) {
     float q[WS::N];
     WS::q(T, E, q);
 #pragma unroll
-    for (int s = 0; s < WS::N; s++) {
-      acc.thr[s] = fminf(acc.thr[s], q[s]);
-      if (q[s] <= acc.thr[s] * (1.f + p.delta[p.ws_perm[s]])) need |= 1u << s;
-    }
+    for (int s = 0; s < WS::N; s++)
+      if (q[s] <= fminf(thr.v[s], q[s]) * (1.f + p.delta[p.ws_perm[s]])) need |= 1u << s;
   }
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
-  if (!need && !par) return;
-  acc.nref++;
+  if (!need && !par) return 0;
   int lam[kMaxN];
   for (int i = 0; i < p.n; i++) lam[i] = dig[wp.cfg.a[i]];
   double T64r, E64;
-  refine64(tb, p, wp.cfg.mask, K, lam, &T64r, &E64);
+  refine64(tb, p, wp.cfg.mask, wp.cfg.k, lam, &T64r, &E64);
   if constexpr (WS::N > 0) {
 #pragma unroll
     for (int s = 0; s < WS::N; s++) {
       if (need >> s & 1u) {
         const double F = objective64(p, T64r, E64, WS::A(s), WS::B(s));
-        BestRec &b = acc.lb[s];
+        BestRec &b = lb[s];
         if (!b.valid || better(F, idx, b.f, b.idx)) {
           b.f = F;
           b.idx = idx;
@@ -178,184 +191,191 @@ __device__ __noinline__ void check_config(const Tables &tb, const DevParams &p, 
   }
   if (par && !stair_dominated(stair, p, T64r, __double2float_rd(__ddiv_rd(E64, p.eseq))))
     emit_candidate(p, stair, idx, T64r, E64, T, E);
+  return 1;
 }
 
-// per-config path for v in [v0, v1) of the current partition, strided by lanes
-template <int L, class WS, int K>
-__device__ __forceinline__ void edge_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                             const WarpPart &wp, LaneAcc<WS> &acc, u64 v0, u64 v1, int lane) {
-  for (u64 v = v0 + lane; v < v1; v += 32) {
-    int dig[K];
-    u64 x = v;
-#pragma unroll
-    for (int b = K - 1; b >= 0; b--) {
-      dig[b] = (int)(x % L);
-      x /= L;
-    }
+// Per-configuration path for v in [v0, v1) of the current partition with
+// stride `step` (lanes interleave with step 32, a single lane uses 1).
+template <class WS>
+__device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, const Stair &stair,
+                                         const WarpPart &wp, Thr<WS> &thr, BestRec *lb, u64 v0, u64 v1,
+                                         int step) {
+  const int k = wp.cfg.k;
+  int nref = 0;
+  for (u64 v = v0; v < v1; v += step) {
+    int dig[kTileMaxG];
     float T = 0.f, E = 0.f;
     double T64 = 0.0;
-#pragma unroll
-    for (int b = 0; b < K; b++) {
-      T = fmaxf(T, wp.gt[b * L + dig[b]]);
-      E += wp.ge[b * L + dig[b]];
-      T64 = fmax(T64, wp.g64[b * L + dig[b]]);
+    for (int b = 0; b < k; b++) {
+      dig[b] = (int)(v >> (2 * (k - 1 - b))) & 3;
+      T = fmaxf(T, wp.gt[b * 4 + dig[b]]);
+      E += wp.ge[b * 4 + dig[b]];
+      T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
-    check_config<L, WS, K>(tb, p, stair, wp, acc, wp.base + v, dig, T, E, T64);
+    if constexpr (WS::N > 0) {
+      float q[WS::N];
+      WS::q(T, E, q);
+#pragma unroll
+      for (int s = 0; s < WS::N; s++) thr.v[s] = fminf(thr.v[s], q[s]);
+    }
+    nref += check_config<WS>(tb, p, stair, wp, thr, lb, wp.base + v, dig, T, E, T64);
   }
+  return nref;
 }
 
-// Full tiles [t0, t1) of this lane (tile t = level digits of groups 0..K-3).
-template <int L, class WS, int K>
-__device__ __forceinline__ void lane_tiles(const Tables &tb, const DevParams &p, const Stair &stair,
-                                           const WarpPart &wp, LaneAcc<WS> &acc, u64 t0, u64 t1) {
-  constexpr int KP = K - 2;  // prefix groups
-  constexpr int L2 = L * L;
-  float At[L], Ae[L], Bt[L], Be[L];
-  double A64[L], B64[L];
-#pragma unroll
-  for (int m = 0; m < L; m++) {
-    At[m] = wp.gt[(K - 2) * L + m];
-    Ae[m] = wp.ge[(K - 2) * L + m];
-    A64[m] = wp.g64[(K - 2) * L + m];
-    Bt[m] = wp.gt[(K - 1) * L + m];
-    Be[m] = wp.ge[(K - 1) * L + m];
-    B64[m] = wp.g64[(K - 1) * L + m];
+// Slow path of one 64-configuration tile (v = vt .. vt+63, k >= 5).
+template <class WS>
+__device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, const Stair &stair,
+                                      const WarpPart &wp, const Thr<WS> thr, BestRec *lb, u64 vt, float Tp,
+                                      float Ep) {
+  const int k = wp.cfg.k;
+  int dig[kTileMaxG];
+  double Tp64 = 0.0;
+  for (int b = 0; b < k - 3; b++) {
+    dig[b] = (int)(vt >> (2 * (k - 1 - b))) & 3;
+    Tp64 = fmax(Tp64, wp.g64[b * 4 + dig[b]]);
   }
-  float minAe = Ae[0], minBe = Be[0];
-  double minA64 = A64[0], minB64 = B64[0];
-#pragma unroll
-  for (int m = 1; m < L; m++) {
-    minAe = fminf(minAe, Ae[m]);
-    minBe = fminf(minBe, Be[m]);
-    minA64 = fmin(minA64, A64[m]);
-    minB64 = fmin(minB64, B64[m]);
-  }
-  // odometer over the prefix digits
-  int dg[KP > 0 ? KP : 1];
-  float PT[KP > 0 ? KP : 1], PE[KP > 0 ? KP : 1];
-  double P64[KP > 0 ? KP : 1];
-  {
-    u64 x = t0;
-#pragma unroll
-    for (int j = KP - 1; j >= 0; j--) {
-      dg[j] = (int)(x % L);
-      x /= L;
-    }
-#pragma unroll
-    for (int j = 0; j < KP; j++) {
-      const float pt = j ? PT[j - 1] : 0.f, pe = j ? PE[j - 1] : 0.f;
-      const double p64 = j ? P64[j - 1] : 0.0;
-      PT[j] = fmaxf(pt, wp.gt[j * L + dg[j]]);
-      PE[j] = pe + wp.ge[j * L + dg[j]];
-      P64[j] = fmax(p64, wp.g64[j * L + dg[j]]);
+  const int ga = (k - 3) * 4, gb = (k - 2) * 4, gc = (k - 1) * 4;
+  int nref = 0;
+  for (int a = 0; a < 4; a++) {
+    const float T1 = fmaxf(Tp, wp.gt[ga + a]), E1 = Ep + wp.ge[ga + a];
+    for (int b = 0; b < 4; b++) {
+      const float T2 = fmaxf(T1, wp.gt[gb + b]), E2 = E1 + wp.ge[gb + b];
+      for (int c = 0; c < 4; c++) {
+        const float T = fmaxf(T2, wp.gt[gc + c]), E = E2 + wp.ge[gc + c];
+        const double T64 = fmax(fmax(fmax(Tp64, wp.g64[ga + a]), wp.g64[gb + b]), wp.g64[gc + c]);
+        dig[k - 3] = a;
+        dig[k - 2] = b;
+        dig[k - 1] = c;
+        nref += check_config<WS>(tb, p, stair, wp, thr, lb, wp.base + vt + a * 16 + b * 4 + c, dig, T, E, T64);
+      }
     }
   }
-  for (u64 t = t0; t < t1; t++) {
-    const float Tp = KP ? PT[KP - 1] : 0.f, Ep = KP ? PE[KP - 1] : 0.f;
-    const double Tp64 = KP ? P64[KP - 1] : 0.0;
-    // ---- score the L^2 configurations of the tile ----
+  return nref;
+}
+
+// exact min fp64 makespan over a tile (its corner), k >= 5
+static __device__ __noinline__ double tile_corner64(const WarpPart &wp, u64 vt, double minC64) {
+  const int k = wp.cfg.k;
+  double t = minC64;
+  for (int b = 0; b < k - 3; b++) t = fmax(t, wp.g64[b * 4 + ((int)(vt >> (2 * (k - 1 - b))) & 3)]);
+  return t;
+}
+
+// All level vectors v in [v0, v1) of the current partition (L = 4).
+// k >= 5: lane = (h, digit of group k-5, digit of group k-4); the warp loop
+// runs over j = digit strings of groups 0..k-6, two per step (h selects);
+// each lane scores the 64-configuration tile of groups k-3..k-1 in registers.
+template <class WS>
+__device__ __forceinline__ int partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
+                                                 WarpPart &wp, Thr<WS> &thr, BestRec *lb, u64 v0, u64 v1,
+                                                 int lane) {
+  const int k = wp.cfg.k;
+  if (k < 5) return edge_configs<WS>(tb, p, stair, wp, thr, lb, v0 + lane, v1, 32);
+  const int nloop = 1 << (2 * (k - 5));
+  for (int j = lane; j < nloop; j += 32) {  // loop-prefix table
+    float T = 0.f, E = 0.f;
+    for (int b = 0; b < k - 5; b++) {
+      const int d = (j >> (2 * (k - 6 - b))) & 3;
+      T = fmaxf(T, wp.gt[b * 4 + d]);
+      E += wp.ge[b * 4 + d];
+    }
+    wp.lp[j] = make_float2(T, E);
+  }
+  __syncwarp();
+  const int h = lane >> 4, l4 = lane & 15;
+  const int ga = (k - 3) * 4, gb = (k - 2) * 4, gc = (k - 1) * 4;
+  const float Tl = fmaxf(wp.gt[(k - 5) * 4 + (l4 >> 2)], wp.gt[(k - 4) * 4 + (l4 & 3)]);
+  const float El = wp.ge[(k - 5) * 4 + (l4 >> 2)] + wp.ge[(k - 4) * 4 + (l4 & 3)];
+  float At[4], Ae[4], Bt[4], Be[4], Ct[4], Ce[4];
+#pragma unroll
+  for (int m = 0; m < 4; m++) {
+    At[m] = wp.gt[ga + m];
+    Ae[m] = wp.ge[ga + m];
+    Bt[m] = wp.gt[gb + m];
+    Be[m] = wp.ge[gb + m];
+    Ct[m] = wp.gt[gc + m];
+    Ce[m] = wp.ge[gc + m];
+  }
+  const float minTin = fmaxf(fmaxf(fminf(fminf(At[0], At[1]), fminf(At[2], At[3])),
+                                   fminf(fminf(Bt[0], Bt[1]), fminf(Bt[2], Bt[3]))),
+                             fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
+  const float minAe = fminf(fminf(Ae[0], Ae[1]), fminf(Ae[2], Ae[3]));
+  const float minBe = fminf(fminf(Be[0], Be[1]), fminf(Be[2], Be[3]));
+  const float minCe = fminf(fminf(Ce[0], Ce[1]), fminf(Ce[2], Ce[3]));
+  const double minC64 = fmax(fmax(fmin(wp.g64[ga], fmin(wp.g64[ga + 1], fmin(wp.g64[ga + 2], wp.g64[ga + 3]))),
+                       fmin(wp.g64[gb], fmin(wp.g64[gb + 1], fmin(wp.g64[gb + 2], wp.g64[gb + 3])))),
+                  fmin(wp.g64[gc], fmin(wp.g64[gc + 1], fmin(wp.g64[gc + 2], wp.g64[gc + 3]))));
+  float mul[WS::N > 0 ? WS::N : 1];
+#pragma unroll
+  for (int s = 0; s < WS::N; s++) mul[s] = 1.f + p.delta[p.ws_perm[s]];
+  const float tlbs = p.tlb_scale_f;
+  int nref = 0;
+  const u64 s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
+  for (u64 st = s_lo; st <= s_hi; st++) {
+    const u64 j = 2 * st + h;
+    if (j >= (u64)nloop) continue;
+    const u64 vt = (j << 10) | ((u64)l4 << 6);
+    if (vt + 64 <= v0 || vt >= v1) continue;
+    const float2 lp = wp.lp[j];
+    const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
+    if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
+      nref += edge_configs<WS>(tb, p, stair, wp, thr, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+      continue;
+    }
     bool hit = false;
+    float cE;
     if constexpr (WS::N > 0) {
       float mq[WS::N];
 #pragma unroll
       for (int s = 0; s < WS::N; s++) mq[s] = __int_as_float(0x7f800000);
 #pragma unroll
-      for (int mu = 0; mu < L; mu++) {
-        const float T1 = fmaxf(Tp, At[mu]), E1 = Ep + Ae[mu];
+      for (int a = 0; a < 4; a++) {
+        const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
 #pragma unroll
-        for (int nu = 0; nu < L; nu++) {
-          const float T = fmaxf(T1, Bt[nu]), E = E1 + Be[nu];
-          float q[WS::N];
-          WS::q(T, E, q);
+        for (int b = 0; b < 4; b++) {
+          const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
 #pragma unroll
-          for (int s = 0; s < WS::N; s++) mq[s] = fminf(mq[s], q[s]);
+          for (int c = 0; c < 4; c++) {
+            const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
+            float q[WS::N];
+            WS::q(T, E, q);
+#pragma unroll
+            for (int s = 0; s < WS::N; s++) mq[s] = fminf(mq[s], q[s]);
+          }
         }
       }
 #pragma unroll
       for (int s = 0; s < WS::N; s++) {
-        acc.thr[s] = fminf(acc.thr[s], mq[s]);
-        hit |= mq[s] <= acc.thr[s] * (1.f + p.delta[p.ws_perm[s]]);
+        thr.v[s] = fminf(thr.v[s], mq[s]);
+        hit |= mq[s] <= thr.v[s] * mul[s];
       }
-    }
-    float cE;
-    if constexpr (WS::N == 0) {  // Pareto only: per-configuration E, min-reduced
+      cE = ((Ep + minAe) + minBe) + minCe;  // = min over the tile of the fp32 E above
+    } else {  // Pareto only: per-configuration E, min-reduced
       cE = __int_as_float(0x7f800000);
 #pragma unroll
-      for (int mu = 0; mu < L; mu++) {
-        const float E1 = Ep + Ae[mu];
+      for (int a = 0; a < 4; a++) {
+        const float E1 = Ep + Ae[a];
 #pragma unroll
-        for (int nu = 0; nu < L; nu++) cE = fminf(cE, E1 + Be[nu]);
+        for (int b = 0; b < 4; b++) {
+          const float E2 = E1 + Be[b];
+#pragma unroll
+          for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
+        }
       }
-    } else {
-      cE = (Ep + minAe) + minBe;  // = min over the tile of the fp32 E above
     }
     if (!hit && p.want_pareto) {
-      const double cT64 = fmax(fmax(Tp64, minA64), minB64);  // exact min T64 over the tile
-      hit = !stair_dominated(stair, p, cT64, cE);
+      if (!stair_dominated_f(stair, p, __fmul_rd(fmaxf(Tp, minTin), tlbs), cE))
+        hit = !stair_dominated(stair, p, tile_corner64(wp, vt, minC64), cE);
     }
-    if (hit) {  // slow path: configuration by configuration
-      int dig[K];
-#pragma unroll
-      for (int j = 0; j < KP; j++) dig[j] = dg[j];
-#pragma unroll
-      for (int mu = 0; mu < L; mu++) {
-#pragma unroll
-        for (int nu = 0; nu < L; nu++) {
-          dig[K - 2] = mu;
-          dig[K - 1] = nu;
-          const float T = fmaxf(fmaxf(Tp, At[mu]), Bt[nu]), E = (Ep + Ae[mu]) + Be[nu];
-          const double T64 = fmax(fmax(Tp64, A64[mu]), B64[nu]);
-          check_config<L, WS, K>(tb, p, stair, wp, acc, wp.base + t * L2 + mu * L + nu, dig, T, E, T64);
-        }
-      }
-    }
-    // ---- advance the odometer ----
-    if constexpr (KP > 0) {
-      int j = KP - 1;
-      while (j >= 0 && ++dg[j] == L) {
-        dg[j] = 0;
-        j--;
-      }
-      if (j < 0) j = 0;
-#pragma unroll
-      for (int jj = 0; jj < KP; jj++) {
-        if (jj >= j) {
-          const float pt = jj ? PT[jj - 1] : 0.f, pe = jj ? PE[jj - 1] : 0.f;
-          const double p64 = jj ? P64[jj - 1] : 0.0;
-          PT[jj] = fmaxf(pt, wp.gt[jj * L + dg[jj]]);
-          PE[jj] = pe + wp.ge[jj * L + dg[jj]];
-          P64[jj] = fmax(p64, wp.g64[jj * L + dg[jj]]);
-        }
-      }
-    }
+    if (hit) nref += tile_slow<WS>(tb, p, stair, wp, thr, lb, vt, Tp, Ep);
   }
+  __syncwarp();
+  return nref;
 }
-
-template <int L, class WS, int K>
-__device__ __forceinline__ void partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                                  const WarpPart &wp, LaneAcc<WS> &acc, u64 v0, u64 v1,
-                                                  int lane) {
-  constexpr u64 L2 = (u64)L * L;
-  if constexpr (K == 1) {
-    edge_configs<L, WS, K>(tb, p, stair, wp, acc, v0, v1, lane);
-  } else {
-    const u64 ta = (v0 + L2 - 1) / L2, tb2 = v1 / L2;
-    if (ta >= tb2) {
-      edge_configs<L, WS, K>(tb, p, stair, wp, acc, v0, v1, lane);
-      return;
-    }
-    edge_configs<L, WS, K>(tb, p, stair, wp, acc, v0, ta * L2, lane);
-    edge_configs<L, WS, K>(tb, p, stair, wp, acc, tb2 * L2, v1, lane);
-    const u64 nt = tb2 - ta, q = nt / 32, r = nt % 32;
-    const u64 my0 = ta + lane * q + (lane < (int)r ? lane : r);
-    const u64 my1 = my0 + q + (lane < (int)r ? 1 : 0);
-    if (my0 < my1) lane_tiles<L, WS, K>(tb, p, stair, wp, acc, my0, my1);
-  }
-}
-
 
 template <int L, class WS>
-__global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
+__global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, p);
   const Tables tb = tables_at(sm, p);
@@ -368,14 +388,14 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
   stair_init(stair);
   __syncthreads();
 
-  LaneAcc<WS> acc;
+  Thr<WS> thr;
+  BestRec lb[WS::N > 0 ? WS::N : 1];
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {
-    acc.thr[s] = __int_as_float(0x7f800000);
-    best_init(acc.lb[s]);
+    thr.v[s] = __int_as_float(0x7f800000);
+    best_init(lb[s]);
   }
-  acc.nref = 0;
-  u64 ncfg = 0, nfeas = 0, stair_ver = 0;
+  u64 ncfg = 0, nfeas = 0, stair_ver = 0, nref = 0;
   const int ul = p.unit_log2, cl = p.chunk_log2;
 
   for (;;) {
@@ -383,14 +403,15 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
     if (lane == 0) unit = atomicAdd(p.ctr + kCtrUnit, 1ull);
     unit = __shfl_sync(0xffffffffu, unit, 0);
     if (unit >= p.n_units) break;
-    const u64 ch = p.first_chunk + (unit >> (cl - ul)) * (u64)p.shard_count;
-    u64 s = (ch << cl) + ((unit & ((1ull << (cl - ul)) - 1)) << ul);
+    const u64 ue = unit * p.unit_stride;
+    const u64 ch = p.first_chunk + (ue >> (cl - ul)) * (u64)p.shard_count;
+    u64 s = (ch << cl) + ((ue & ((1ull << (cl - ul)) - 1)) << ul);
     u64 e = s + (1ull << ul);
     s = s > p.lo ? s : p.lo;
     e = e < p.hi ? e : p.hi;
     if (s >= e) continue;
 #pragma unroll
-    for (int w = 0; w < WS::N; w++) acc.thr[w] = fminf(acc.thr[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
+    for (int w = 0; w < WS::N; w++) thr.v[w] = fminf(thr.v[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
     if (p.want_pareto) {
       const u64 v = __ldcg(p.ctr + kCtrStairVer);
       if (v != stair_ver) {
@@ -403,7 +424,15 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
+    u64 ver_pref = p.want_pareto ? __ldcg(p.ctr + kCtrStairVer) : 0;
     for (;;) {
+      if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
+        if (ver_pref != stair_ver) {
+          stair_ver = ver_pref;
+          stair_merge(stair, p);
+        }
+        ver_pref = __ldcg(p.ctr + kCtrStairVer);
+      }
       const u64 base = wp.base, Pn = wp.cfg.Pn;
       const int k = wp.cfg.k;
       const u64 v0 = s > base ? s - base : 0, v1 = e - base < Pn ? e - base : Pn;
@@ -423,16 +452,7 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
           wp.g64[b * L + mu] = t64;
         }
         __syncwarp();
-        switch (k) {
-          case 1: partition_configs<L, WS, 1>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 2: partition_configs<L, WS, 2>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 3: partition_configs<L, WS, 3>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 4: partition_configs<L, WS, 4>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 5: partition_configs<L, WS, 5>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 6: partition_configs<L, WS, 6>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          case 7: partition_configs<L, WS, 7>(tb, p, stair, wp, acc, v0, v1, lane); break;
-          default: partition_configs<L, WS, 8>(tb, p, stair, wp, acc, v0, v1, lane); break;
-        }
+        nref += partition_configs<WS>(tb, p, stair, wp, thr, lb, v0, v1, lane);
       }
       __syncwarp();
       if (base + Pn >= e) break;
@@ -447,16 +467,15 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
     }
 #pragma unroll
     for (int w = 0; w < WS::N; w++) {
-      float t = acc.thr[w];
+      float t = thr.v[w];
 #pragma unroll
       for (int o = 16; o; o >>= 1) t = fminf(t, __shfl_xor_sync(0xffffffffu, t, o));
-      acc.thr[w] = t;
+      thr.v[w] = t;
       if (lane == 0 && t < __uint_as_float(__ldcg(p.thr + p.ws_perm[w])))
         atomicMin(p.thr + p.ws_perm[w], __float_as_uint(t));
     }
   }
   // ---- reductions ----
-  u64 nref = acc.nref;
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
     ncfg += __shfl_xor_sync(0xffffffffu, ncfg, o);
@@ -470,8 +489,8 @@ __global__ void __launch_bounds__(kTileThreads) k_tile(const DevParams p) {
   }
 #pragma unroll
   for (int w = 0; w < WS::N; w++) {
-    warp_best(acc.lb[w]);
-    if (lane == 0) red[warp * kMaxW + w] = acc.lb[w];
+    warp_best(lb[w]);
+    if (lane == 0) red[warp * kMaxW + w] = lb[w];
   }
   __syncthreads();
   if (threadIdx.x < WS::N) {

@@ -53,7 +53,7 @@ bool tile_eligible(DevParams &dp, TileLaunch *tl) {
 }
 
 cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
-                        cudaEvent_t e2, int *grid) {
+                        cudaEvent_t e2, int *grid, bool fixed_units) {
   cudaError_t err = cudaFuncSetAttribute(tl.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tl.smem);
   if (err != cudaSuccess) return err;
   int occ = 0;
@@ -62,12 +62,15 @@ cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream
   if (occ < 1) return cudaErrorInvalidConfiguration;
   *grid = std::min(4096, nsm * occ);
   // unit size: ~16 units per warp over the search, 2^12 .. 2^chunk_log2 configs
-  const uint64_t range = dp.n_owned << dp.chunk_log2;
-  const uint64_t warps = (uint64_t)(*grid) * kTileWarps;
-  int ul = 12;
-  while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 16) ul++;
-  dp.unit_log2 = ul;
-  dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+  if (!fixed_units) {
+    const uint64_t range = dp.n_owned << dp.chunk_log2;
+    const uint64_t warps = (uint64_t)(*grid) * kTileWarps;
+    int ul = 12;
+    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 16) ul++;
+    dp.unit_log2 = ul;
+    dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+    dp.unit_stride = 1;
+  }
   void *args[] = {(void *)&dp};
   cudaEventRecord(e1, st);
   err = cudaLaunchKernel(tl.fn, *grid, kTileThreads, args, tl.smem, st);
