@@ -456,7 +456,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   // the full search; pass 2 only after a candidate-buffer overflow.
   const DevParams dp_full = dp;
   const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
-                    (dp.n_owned << (dp.chunk_log2 - 12)) >= (uint64_t)nsm * 64 * 16;
+                    (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 26);  // >= 2^38 configs
   for (int pass = seed ? 0 : 1; pass < 3; pass++) {
     dp = dp_full;
     if (pass == 0) {
