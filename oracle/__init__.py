@@ -26,6 +26,7 @@ from . import counts  # noqa: F401
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "enum.c")
+_SRCS = [_SRC, os.path.join(_HERE, "dpcert.c")]
 _lib = None
 
 ORACLE_CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-msse2",
@@ -33,9 +34,9 @@ ORACLE_CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-msse2",
 
 
 def build(force: bool = False) -> str:
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+    if force or not os.path.exists(_SO) or any(os.path.getmtime(_SO) < os.path.getmtime(x) for x in _SRCS):
         tmp = _SO + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", *ORACLE_CFLAGS, "-o", tmp, _SRC])
+        subprocess.check_call(["gcc", *ORACLE_CFLAGS, "-o", tmp, *_SRCS])
         os.replace(tmp, _SO)
     return _SO
 
@@ -230,3 +231,21 @@ def score(prof, q, rgs, digits):
 
 def objective(tseq, eseq, T, E, a, b) -> float:
     return lib().oracle_objective(tseq, eseq, T, E, a, b)
+
+
+def dp_certificate(prof, q, cap: int = 1 << 20):
+    """O3 (dpcert.c): exact Pareto-front values [(T, E)] (T ascending) of the
+    whole PER_GPU space and the exact optimum F per weight (max over the
+    front, canonical fp64).  Values only, no indices."""
+    assert q.scope == 1, "certificate covers PER_GPU scope"
+    pk = _Pack(prof, q)
+    ot = (C.c_double * cap)()
+    oe = (C.c_double * cap)()
+    lev = (C.c_int * len(pk.lev_idx))(*pk.lev_idx)
+    nf = lib().oracle_dpcert(C.byref(pk.P), q.n, q.g, min(q.c, q.n), len(q.levels), lev, ot, oe, cap)
+    if nf < 0:
+        raise RuntimeError("certificate capacity / size")
+    front = [(ot[i], oe[i]) for i in range(nf)]
+    ts, es = constants(prof, q)
+    best = [max(objective(ts, es, T, E, a, b) for T, E in front) if front else None for a, b in q.weights]
+    return dict(front=front, best=best, tseq=ts, eseq=es)

@@ -170,3 +170,30 @@ def test_c3_full_size_properties():
             assert r["best"][0][1] < b.score64 or (r["best"][0][1] == b.score64 and r["best"][0][0] >= b.index)
         for _, T, E in r["pareto"]:
             assert any(t2 <= T and e2 <= E for t2, e2 in front)
+
+
+def _certificate(name):
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"{name}_certificate.json")))
+    front = [(float.fromhex(t), float.fromhex(e)) for t, e in g["front_T_E"]]
+    best = [float.fromhex(b) for b in g["best_score64"]]
+    return front, best
+
+
+@pytest.mark.parametrize("name", ["c3", "c4"])
+def test_full_space_vs_dp_certificate(name):
+    """Full c3 / c4 search (c4: 2.07e14 configurations, ~70 s on one B200) in
+    the bench's launch configuration vs the O3 subset-DP certificate
+    (tests/golden/<cfg>_certificate.json, written by oracle/make_certificates.py):
+    the Pareto front values and the optimum of every weight must be bitwise
+    equal; every returned index is re-scored by the oracle."""
+    prof, q = config(name)
+    front, best = _certificate(name)
+    res = S.Scheduler(prof).search(q)
+    assert res.stats["n_configs"] == S.count(q)
+    assert [(p.makespan_s, p.energy_j) for p in res.pareto] == front
+    assert [b.score64 for b in res.best] == best
+    for p in list(res.pareto) + list(res.best):
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
+        assert ok and (T, E) == (p.makespan_s, p.energy_j)
