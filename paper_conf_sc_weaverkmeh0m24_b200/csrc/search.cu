@@ -478,6 +478,9 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     if (tile_eligible(dp, &tl)) {
       path = 1;
       CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
+    } else if (dfs_eligible(dp, &tl)) {
+      path = 2;
+      CK(launch_dfs(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
     } else {
       const size_t smem = ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(BestRec) * kWarps * kMaxW;
       CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));

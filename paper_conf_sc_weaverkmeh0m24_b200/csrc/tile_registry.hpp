@@ -14,6 +14,8 @@ struct WS_11;
 struct WS_10;
 struct WS_01;
 struct WS_11_21;
+struct WS_SWEEP;
+struct WS_C1;
 
 template <int L, class WS>
 const void *tile_fn();
@@ -29,6 +31,9 @@ constexpr int kTileMaxL = 4;
 constexpr int kTileMaxG = 8;
 size_t tile_smem_bytes(const DevParams &dp);
 bool tile_eligible(DevParams &dp, TileLaunch *tl);
+bool dfs_eligible(DevParams &dp, TileLaunch *tl);
+cudaError_t launch_dfs(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                       cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
                         cudaEvent_t e2, int *grid, bool fixed_units);
 

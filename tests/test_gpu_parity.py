@@ -197,3 +197,33 @@ def test_full_space_vs_dp_certificate(name):
     for p in list(res.pareto) + list(res.best):
         ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
         assert ok and (T, E) == (p.makespan_s, p.energy_j)
+
+
+@pytest.mark.parametrize("n,g,c,ws,seed", [
+    (9, 4, 3, ((1, 0), (3, 1), (2, 1), (1, 1), (1, 2), (1, 3), (0, 1)), 1),
+    (10, 5, 2, ((1, 1),), 2), (8, 8, 4, ((1, 1), (2, 1)), 3), (11, 4, 3, (), 4), (7, 3, 4, ((1, 0),), 5),
+])
+def test_partition_kernel_path(n, g, c, ws, seed):
+    """L = 1 spaces (every configuration is a partition) run on the partition
+    kernel (kernel_path 2) and must equal the oracle exactly."""
+    prof = make_profile(n, levels=(100,), seed=seed)
+    q = Query(n, g, c, (100,), PER_GPU, ws, True)
+    res = S.Scheduler(prof).search(q)
+    assert res.stats["kernel_path"] == 2
+    check(res, oracle.search(prof, q), q)
+    lo = S.count(q) // 3
+    qw = q.with_range(lo, lo + 12345)
+    res = S.Scheduler(prof).search(qw)
+    check(res, oracle.search(prof, qw), qw)
+
+
+@pytest.mark.parametrize("n,g,c,ws,seed", [
+    (8, 4, 8, ((1, 1),), 1), (9, 6, 3, ((1, 1), (2, 1)), 2), (7, 7, 7, (), 3), (9, 8, 9, ((1, 0),), 4),
+])
+def test_tile_kernel_path(n, g, c, ws, seed):
+    """L = 4 PER_GPU spaces run on the tile kernel (kernel_path 1)."""
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, (25, 50, 75, 100), PER_GPU, ws, True)
+    res = S.Scheduler(prof).search(q)
+    assert res.stats["kernel_path"] == 1
+    check(res, oracle.search(prof, q), q)

@@ -1,0 +1,45 @@
+"""O3 (subset-DP certificate) pinned against O1 (full enumeration) on every
+PER_GPU space small enough to enumerate: Pareto-front values and the
+optimum of every weight must be bitwise equal.  The stored c3/c4
+certificates (tests/golden) must be reproducible from oracle/ alone."""
+import json
+import os
+
+import pytest
+
+import oracle
+from synth import Query, config, make_profile, PER_GPU
+
+W = ((1, 1), (2, 1), (1, 0), (0, 1), (1, 3))
+
+
+@pytest.mark.parametrize("n,g,c,levels,seed", [
+    (5, 2, 3, (50, 100), 1), (6, 3, 3, (25, 50, 100), 2), (7, 4, 7, (50, 100), 3),
+    (8, 3, 3, (25, 50, 75, 100), 4), (9, 4, 4, (50, 100), 5), (8, 8, 8, (100,), 6),
+    (9, 5, 2, (25, 100), 7),
+])
+def test_certificate_equals_enumeration(n, g, c, levels, seed):
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, levels, PER_GPU, W, True)
+    r = oracle.search(prof, q)
+    cert = oracle.dp_certificate(prof, q)
+    assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
+    assert [b[1] for b in r["best"]] == cert["best"]
+
+
+def test_certificate_handles_infeasible_groups():
+    prof = make_profile(6, levels=(50, 100), seed=3, archetypes=[11, 2, 0, 12, 5, 1])
+    q = Query(6, 3, 6, (50, 100), PER_GPU, W, True)
+    r = oracle.search(prof, q)
+    cert = oracle.dp_certificate(prof, q)
+    assert r["nfeasible"] < r["nconfigs"]
+    assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
+
+
+@pytest.mark.parametrize("name", ["c3", "c4"])
+def test_golden_certificates_reproduce(name):
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"{name}_certificate.json")))
+    prof, q = config(name)
+    cert = oracle.dp_certificate(prof, q)
+    assert [[t.hex(), e.hex()] for t, e in cert["front"]] == g["front_T_E"]
+    assert [b.hex() for b in cert["best"]] == g["best_score64"]
