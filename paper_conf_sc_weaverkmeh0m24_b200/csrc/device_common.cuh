@@ -251,6 +251,44 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
   for (int i = jb + 1; i < hi; i++) atomicMin(s.pm + i, vb);
 }
 
+// fp32 + exact fp64 makespan of group `m` with every member at level mu
+__device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p, uint32_t m, int mu,
+                                           float &t32, float &e32, double &t64) {
+  const int L = p.L;
+  float U = 0.f, B = 0.f, D = 0.f;
+  double U64 = 0.0, B64 = 0.0;
+  for (uint32_t mm = m; mm; mm &= mm - 1) {
+    const int r = (__ffs(mm) - 1) * L + mu;
+    U += tb.u[r];
+    B += tb.bw[r];
+    D += tb.dh[r];
+    U64 = __dadd_rn(U64, (double)tb.u[r]);
+    B64 = __dadd_rn(B64, (double)tb.bw[r]);
+  }
+  const float cg = fmaxf(fmaxf(1.f, U), B);
+  double c = 1.0;
+  if (U64 > c) c = U64;
+  if (B64 > c) c = B64;
+  float Tg = 0.f;
+  double Tg64 = 0.0;
+  for (uint32_t mm = m; mm; mm &= mm - 1) {
+    const int i = __ffs(mm) - 1, ri = i * L + mu;
+    float s = 1.f;
+    double s64 = 1.0;
+    for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) {
+      const float dv = tb.d[ri * p.ds + (__ffs(m2) - 1) * L + mu];
+      s += dv;
+      s64 = __dadd_rn(s64, (double)dv);
+    }
+    Tg = fmaxf(Tg, tb.th[ri] * s * cg);
+    const double tau = __dmul_rn(__dmul_rn((double)tb.traw[ri], s64), c);
+    if (tau > Tg64) Tg64 = tau;
+  }
+  t32 = Tg;
+  e32 = p.phat * Tg + D;
+  t64 = Tg64;
+}
+
 // ------------------------------------------------------------ DP walk (RGS state)
 struct LaneCfg {
   int8_t a[kMaxN];

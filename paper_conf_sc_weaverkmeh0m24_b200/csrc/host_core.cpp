@@ -425,6 +425,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   for (int w = 0; w < q.nw; w++) {
     const double eta = q.wa[w] * eT + q.wb[w] * eE + (q.wa[w] + q.wb[w] + 2.0) * u;
     dp->delta[w] = (float)(4.0 * eta);
+    dp->mul[w] = 1.f + dp->delta[w];
   }
   dp->gamma = (float)(2.0 * std::max(eT, eE) + 4.0 * u);
   dp->tlb_scale = std::nextafter(tseq / (1.0 + 2.0 * eT), 0.0);
@@ -510,6 +511,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->n_units = dp->n_owned << (dp->chunk_log2 - dp->unit_log2);
   dp->unit_stride = 1;
   dp->cand_cap = q.cand_cap;
+  dp->gtab_ok = ((uint64_t)L << n) * sizeof(GroupRec) <= ((uint64_t)256 << 20);
   {  // interleave lanes when partitions hold enough level vectors to keep lanes together
     double per = 1.0;
     const int nd = q.scope == SCHED_PER_CLIENT ? n : std::min(q.g, n);

@@ -65,6 +65,7 @@ struct DevParams {
   float delta[kMaxW];       // fp32 screen margin per weight
   float gamma;              // Pareto "surely dominated" margin
   int ws_perm[kMaxW];       // tile kernel: compile-time weight slot -> query weight index
+  float mul[kMaxW];         // 1 + delta[w]
   double tlb_scale;         // T_seq / (1 + 2 eps_T) rounded down: T64 >= T32hat * tlb_scale
   float tlb_scale_f;        // the same, as a float rounded down
   float phat;               // P_s * T_seq / E_seq
@@ -92,6 +93,8 @@ struct DevParams {
   unsigned char *cand;         // [cand_cap] CandRec
   uint32_t cand_cap;
   unsigned char *out;          // finalize output area
+  const unsigned char *gtab;   // [2^n][L] GroupRec: fp32/fp64 group tuples (nullptr: compute)
+  int gtab_ok;                 // workspace holds a group table for this query
 };
 
 enum {
@@ -113,6 +116,11 @@ struct BestRec {      // 48 B
   unsigned long long idx;
   float t32, e32;     // normalised fp32 T/T_seq, E/E_seq of the hot loop
   int valid, pad;
+};
+
+struct GroupRec {     // 16 B: one (group mask, level) tuple; t32 = +inf marks memory-infeasible
+  float t32, e32;     // normalised fp32 T_g / T_seq, E_g / E_seq of the hot loop
+  double t64;         // exact canonical fp64 T_g
 };
 
 struct CandRec {      // 32 B

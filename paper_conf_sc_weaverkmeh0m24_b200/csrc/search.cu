@@ -221,6 +221,32 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
   }
 }
 
+// ------------------------------------------------------------ group table
+// Every (group mask, level) tuple of the query, once per search: fp32
+// normalised T_g, E_g and the exact fp64 T_g (t32 = +inf: memory-infeasible
+// or more than C members).  L2-resident; replaces per-partition evaluation.
+__global__ void __launch_bounds__(256) k_groups(const DevParams p, GroupRec *gtab) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  stage_blob(sm, p);
+  const Tables tb = tables_at(sm, p);
+  const unsigned long long total = (unsigned long long)p.L << p.n;
+  for (unsigned long long id = blockIdx.x * (unsigned long long)blockDim.x + threadIdx.x; id < total;
+       id += (unsigned long long)gridDim.x * blockDim.x) {
+    const uint32_t m = (uint32_t)(id / p.L);
+    const int mu = (int)(id % p.L);
+    GroupRec r;
+    r.t32 = __int_as_float(0x7f800000);
+    r.e32 = 0.f;
+    r.t64 = __longlong_as_double(0x7ff0000000000000ll);
+    if (m != 0 && __popc(m) <= p.c) {
+      long long M = 0;
+      for (uint32_t mm = m; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
+      if (M <= (long long)p.mem_cap) group_eval(tb, p, m, mu, r.t32, r.e32, r.t64);
+    }
+    gtab[id] = r;
+  }
+}
+
 // ------------------------------------------------------------ init / finalize
 // keep = 0: fresh search; 1: seeded re-run after overflow (keep staircase +
 // thresholds, drop candidates); 2: after the seed pass (keep staircase,
@@ -373,7 +399,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, blob, slots, cand, surv, keep, out, total;
+  size_t ctr, thr, stv, stp, blob, slots, cand, surv, keep, out, gtab, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -395,6 +421,7 @@ WsLayout layout(const DevParams &dp) {
   L.surv = take(4 * (size_t)dp.cand_cap);
   L.keep = take(4 * (size_t)dp.cand_cap);
   L.out = take(sizeof(BestRec) * kMaxW + sizeof(CandRec) * (size_t)kFrontCap);
+  L.gtab = take(dp.gtab_ok ? sizeof(GroupRec) * ((size_t)dp.L << dp.n) : 0);
   L.total = (o + 255) / 256 * 256;
   return L;
 }
@@ -436,6 +463,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.slots = ws + L.slots;
   dp.cand = ws + L.cand;
   dp.out = ws + L.out;
+  dp.gtab = dp.gtab_ok ? ws + L.gtab : nullptr;
   int dev = 0, nsm = 0;
   CK(cudaGetDevice(&dev));
   CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
@@ -454,6 +482,21 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   // pass 0: seed pass over a sample of in-range units (2^12 configs each,
   // spread over the shard) that fills the staircase and thresholds; pass 1:
   // the full search; pass 2 only after a candidate-buffer overflow.
+  if (dp.gtab_ok) {  // group-tuple table (part of the search: counted in search_ms)
+    const size_t gsm = (dp.blob_bytes + 15) & ~15u;
+    CK(cudaFuncSetAttribute(k_groups, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gsm));
+    const unsigned long long tot = (unsigned long long)dp.L << dp.n;
+    const int gb = (int)std::min<unsigned long long>((tot + 255) / 256, (unsigned long long)nsm * 8);
+    CK(cudaEventRecord(e1, st));
+    k_groups<<<gb, 256, gsm, st>>>(dp, (GroupRec *)(ws + L.gtab));
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(e2, st));
+    CK(cudaStreamSynchronize(st));
+    float gms = 0.f;
+    CK(cudaEventElapsedTime(&gms, e1, e2));
+    search_ms += gms;
+    launches++;
+  }
   const DevParams dp_full = dp;
   const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
                     (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 26);  // >= 2^38 configs

@@ -91,44 +91,6 @@ struct WarpPart {
   float2 lp[64];  // loop-prefix (max T, sum E) over groups 0..k-6, one entry per digit string
 };
 
-// fp32 + exact fp64 makespan of group `m` with every member at level mu
-__device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p, uint32_t m, int mu,
-                                           float &t32, float &e32, double &t64) {
-  const int L = p.L;
-  float U = 0.f, B = 0.f, D = 0.f;
-  double U64 = 0.0, B64 = 0.0;
-  for (uint32_t mm = m; mm; mm &= mm - 1) {
-    const int r = (__ffs(mm) - 1) * L + mu;
-    U += tb.u[r];
-    B += tb.bw[r];
-    D += tb.dh[r];
-    U64 = __dadd_rn(U64, (double)tb.u[r]);
-    B64 = __dadd_rn(B64, (double)tb.bw[r]);
-  }
-  const float cg = fmaxf(fmaxf(1.f, U), B);
-  double c = 1.0;
-  if (U64 > c) c = U64;
-  if (B64 > c) c = B64;
-  float Tg = 0.f;
-  double Tg64 = 0.0;
-  for (uint32_t mm = m; mm; mm &= mm - 1) {
-    const int i = __ffs(mm) - 1, ri = i * L + mu;
-    float s = 1.f;
-    double s64 = 1.0;
-    for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) {
-      const float dv = tb.d[ri * p.ds + (__ffs(m2) - 1) * L + mu];
-      s += dv;
-      s64 = __dadd_rn(s64, (double)dv);
-    }
-    Tg = fmaxf(Tg, tb.th[ri] * s * cg);
-    const double tau = __dmul_rn(__dmul_rn((double)tb.traw[ri], s64), c);
-    if (tau > Tg64) Tg64 = tau;
-  }
-  t32 = Tg;
-  e32 = p.phat * Tg + D;
-  t64 = Tg64;
-}
-
 template <class WS>
 struct Thr {
   float v[WS::N > 0 ? WS::N : 1];
@@ -151,11 +113,12 @@ __device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParam
 }
 
 // One configuration of the current partition (level digits dig[0..k-1],
-// exact T64, fp32 T/E): per-weight screen, Pareto screen, fp64 refine,
-// record.  Out of line (slow path).  Returns 1 if it issued a refine.
+// exact T64, fp32 T/E): per-weight screen against the lane's thresholds
+// (thr: shared-memory copy), Pareto screen, fp64 refine, record.  Out of
+// line (slow path).  Returns 1 if it issued a refine.
 template <class WS>
 __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, const Stair &stair,
-                                         const WarpPart &wp, const Thr<WS> thr, BestRec *lb, u64 idx,
+                                         const WarpPart &wp, const float *thr, BestRec *lb, u64 idx,
                                          const int *dig, float T, float E, double T64) {
   unsigned need = 0;
   if constexpr (WS::N > 0) {
@@ -163,7 +126,7 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
     WS::q(T, E, q);
 #pragma unroll
     for (int s = 0; s < WS::N; s++)
-      if (q[s] <= fminf(thr.v[s], q[s]) * (1.f + p.delta[p.ws_perm[s]])) need |= 1u << s;
+      if (q[s] <= fminf(thr[s], q[s]) * p.mul[p.ws_perm[s]]) need |= 1u << s;
   }
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
@@ -196,13 +159,14 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
 
 // Per-configuration path for v in [v0, v1) of the current partition with
 // stride `step` (lanes interleave with step 32, a single lane uses 1).
+// thr is the lane's shared-memory threshold copy (updated here).
 template <class WS>
 __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                         const WarpPart &wp, Thr<WS> &thr, BestRec *lb, u64 v0, u64 v1,
+                                         const WarpPart &wp, float *thr, BestRec *lb, uint32_t v0, uint32_t v1,
                                          int step) {
   const int k = wp.cfg.k;
   int nref = 0;
-  for (u64 v = v0; v < v1; v += step) {
+  for (uint32_t v = v0; v < v1; v += step) {
     int dig[kTileMaxG];
     float T = 0.f, E = 0.f;
     double T64 = 0.0;
@@ -216,18 +180,20 @@ __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, c
       float q[WS::N];
       WS::q(T, E, q);
 #pragma unroll
-      for (int s = 0; s < WS::N; s++) thr.v[s] = fminf(thr.v[s], q[s]);
+      for (int s = 0; s < WS::N; s++) thr[s] = fminf(thr[s], q[s]);
     }
     nref += check_config<WS>(tb, p, stair, wp, thr, lb, wp.base + v, dig, T, E, T64);
   }
   return nref;
 }
 
-// Slow path of one 64-configuration tile (v = vt .. vt+63, k >= 5).
+// Slow path of one 64-configuration tile (v = vt .. vt+63, k >= 5), with
+// hierarchical exact Pareto corners (per a, then per (a, b)) before the
+// per-configuration checks.
 template <class WS>
 __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, const Stair &stair,
-                                      const WarpPart &wp, const Thr<WS> thr, BestRec *lb, u64 vt, float Tp,
-                                      float Ep) {
+                                      const WarpPart &wp, const float *thr, BestRec *lb, uint32_t vt, float Tp,
+                                      float Ep, bool arg_hit) {
   const int k = wp.cfg.k;
   int dig[kTileMaxG];
   double Tp64 = 0.0;
@@ -236,14 +202,22 @@ __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, cons
     Tp64 = fmax(Tp64, wp.g64[b * 4 + dig[b]]);
   }
   const int ga = (k - 3) * 4, gb = (k - 2) * 4, gc = (k - 1) * 4;
+  const double minC64 = fmin(fmin(wp.g64[gc], wp.g64[gc + 1]), fmin(wp.g64[gc + 2], wp.g64[gc + 3]));
+  const double minB64 = fmin(fmin(wp.g64[gb], wp.g64[gb + 1]), fmin(wp.g64[gb + 2], wp.g64[gb + 3]));
+  const float minCe = fminf(fminf(wp.ge[gc], wp.ge[gc + 1]), fminf(wp.ge[gc + 2], wp.ge[gc + 3]));
+  const float minBe = fminf(fminf(wp.ge[gb], wp.ge[gb + 1]), fminf(wp.ge[gb + 2], wp.ge[gb + 3]));
   int nref = 0;
   for (int a = 0; a < 4; a++) {
     const float T1 = fmaxf(Tp, wp.gt[ga + a]), E1 = Ep + wp.ge[ga + a];
+    const double A64 = fmax(Tp64, wp.g64[ga + a]);
+    if (!arg_hit && stair_dominated(stair, p, fmax(fmax(A64, minB64), minC64), (E1 + minBe) + minCe)) continue;
     for (int b = 0; b < 4; b++) {
       const float T2 = fmaxf(T1, wp.gt[gb + b]), E2 = E1 + wp.ge[gb + b];
+      const double B64 = fmax(A64, wp.g64[gb + b]);
+      if (!arg_hit && stair_dominated(stair, p, fmax(B64, minC64), E2 + minCe)) continue;
       for (int c = 0; c < 4; c++) {
         const float T = fmaxf(T2, wp.gt[gc + c]), E = E2 + wp.ge[gc + c];
-        const double T64 = fmax(fmax(fmax(Tp64, wp.g64[ga + a]), wp.g64[gb + b]), wp.g64[gc + c]);
+        const double T64 = fmax(B64, wp.g64[gc + c]);
         dig[k - 3] = a;
         dig[k - 2] = b;
         dig[k - 1] = c;
@@ -255,7 +229,7 @@ __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, cons
 }
 
 // exact min fp64 makespan over a tile (its corner), k >= 5
-static __device__ __noinline__ double tile_corner64(const WarpPart &wp, u64 vt, double minC64) {
+static __device__ __noinline__ double tile_corner64(const WarpPart &wp, uint32_t vt, double minC64) {
   const int k = wp.cfg.k;
   double t = minC64;
   for (int b = 0; b < k - 3; b++) t = fmax(t, wp.g64[b * 4 + ((int)(vt >> (2 * (k - 1 - b))) & 3)]);
@@ -268,10 +242,17 @@ static __device__ __noinline__ double tile_corner64(const WarpPart &wp, u64 vt, 
 // each lane scores the 64-configuration tile of groups k-3..k-1 in registers.
 template <class WS>
 __device__ __forceinline__ int partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                                 WarpPart &wp, Thr<WS> &thr, BestRec *lb, u64 v0, u64 v1,
-                                                 int lane) {
+                                                 WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
+                                                 uint32_t v0, uint32_t v1, int lane) {
   const int k = wp.cfg.k;
-  if (k < 5) return edge_configs<WS>(tb, p, stair, wp, thr, lb, v0 + lane, v1, 32);
+  if (k < 5) {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+    const int r = edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
+#pragma unroll
+    for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+    return r;
+  }
   const int nloop = 1 << (2 * (k - 5));
   for (int j = lane; j < nloop; j += 32) {  // loop-prefix table
     float T = 0.f, E = 0.f;
@@ -303,24 +284,23 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
   const float minAe = fminf(fminf(Ae[0], Ae[1]), fminf(Ae[2], Ae[3]));
   const float minBe = fminf(fminf(Be[0], Be[1]), fminf(Be[2], Be[3]));
   const float minCe = fminf(fminf(Ce[0], Ce[1]), fminf(Ce[2], Ce[3]));
-  const double minC64 = fmax(fmax(fmin(wp.g64[ga], fmin(wp.g64[ga + 1], fmin(wp.g64[ga + 2], wp.g64[ga + 3]))),
-                       fmin(wp.g64[gb], fmin(wp.g64[gb + 1], fmin(wp.g64[gb + 2], wp.g64[gb + 3])))),
-                  fmin(wp.g64[gc], fmin(wp.g64[gc + 1], fmin(wp.g64[gc + 2], wp.g64[gc + 3]))));
-  float mul[WS::N > 0 ? WS::N : 1];
-#pragma unroll
-  for (int s = 0; s < WS::N; s++) mul[s] = 1.f + p.delta[p.ws_perm[s]];
-  const float tlbs = p.tlb_scale_f;
+  const double mc64 = fmax(fmax(fmin(fmin(wp.g64[gb], wp.g64[gb + 1]), fmin(wp.g64[gb + 2], wp.g64[gb + 3])),
+                                fmin(fmin(wp.g64[gc], wp.g64[gc + 1]), fmin(wp.g64[gc + 2], wp.g64[gc + 3]))),
+                           fmin(fmin(wp.g64[ga], wp.g64[ga + 1]), fmin(wp.g64[ga + 2], wp.g64[ga + 3])));
   int nref = 0;
-  const u64 s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
-  for (u64 st = s_lo; st <= s_hi; st++) {
-    const u64 j = 2 * st + h;
-    if (j >= (u64)nloop) continue;
-    const u64 vt = (j << 10) | ((u64)l4 << 6);
-    if (vt + 64 <= v0 || vt >= v1) continue;
+  const uint32_t s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
+  for (uint32_t st = s_lo; st <= s_hi; st++) {
+    const uint32_t j = 2 * st + h;
+    const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
+    if (j >= (uint32_t)nloop || vt + 64 <= v0 || vt >= v1) continue;
     const float2 lp = wp.lp[j];
     const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
     if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-      nref += edge_configs<WS>(tb, p, stair, wp, thr, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+#pragma unroll
+      for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+      nref += edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+#pragma unroll
+      for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
       continue;
     }
     bool hit = false;
@@ -348,9 +328,10 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
 #pragma unroll
       for (int s = 0; s < WS::N; s++) {
         thr.v[s] = fminf(thr.v[s], mq[s]);
-        hit |= mq[s] <= thr.v[s] * mul[s];
+        hit |= mq[s] <= thr.v[s] * p.mul[p.ws_perm[s]];
       }
-      cE = ((Ep + minAe) + minBe) + minCe;  // = min over the tile of the fp32 E above
+      // min over the tile of the fp32 E above ((Ep + a) + b) + c is monotone in each term
+      cE = ((Ep + minAe) + minBe) + minCe;
     } else {  // Pareto only: per-configuration E, min-reduced
       cE = __int_as_float(0x7f800000);
 #pragma unroll
@@ -364,18 +345,21 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         }
       }
     }
-    if (!hit && p.want_pareto) {
-      if (!stair_dominated_f(stair, p, __fmul_rd(fmaxf(Tp, minTin), tlbs), cE))
-        hit = !stair_dominated(stair, p, tile_corner64(wp, vt, minC64), cE);
+    bool par = false;
+    if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(fmaxf(Tp, minTin), p.tlb_scale_f), cE))
+      par = !stair_dominated(stair, p, tile_corner64(wp, vt, mc64), cE);
+    if (hit || par) {
+#pragma unroll
+      for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+      nref += tile_slow<WS>(tb, p, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
     }
-    if (hit) nref += tile_slow<WS>(tb, p, stair, wp, thr, lb, vt, Tp, Ep);
   }
   __syncwarp();
   return nref;
 }
 
 template <int L, class WS>
-__global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
+__global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, p);
   const Tables tb = tables_at(sm, p);
@@ -385,6 +369,8 @@ __global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
   WarpPart *wps = (WarpPart *)(after + 12 * kBuckets);
   WarpPart &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kTileWarps);
+  float *thr_sm = (float *)(red + kTileWarps * kMaxW) + threadIdx.x * kMaxW;
+  const GroupRec *gtab = (const GroupRec *)p.gtab;
   stair_init(stair);
   __syncthreads();
 
@@ -395,7 +381,8 @@ __global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
     thr.v[s] = __int_as_float(0x7f800000);
     best_init(lb[s]);
   }
-  u64 ncfg = 0, nfeas = 0, stair_ver = 0, nref = 0;
+  u64 ncfg = 0, nfeas = 0, stair_ver = 0;
+  int nref = 0;
   const int ul = p.unit_log2, cl = p.chunk_log2;
 
   for (;;) {
@@ -433,27 +420,28 @@ __global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
         }
         ver_pref = __ldcg(p.ctr + kCtrStairVer);
       }
-      const u64 base = wp.base, Pn = wp.cfg.Pn;
+      const u64 base = wp.base;
+      const uint32_t Pn = (uint32_t)wp.cfg.Pn;
       const int k = wp.cfg.k;
-      const u64 v0 = s > base ? s - base : 0, v1 = e - base < Pn ? e - base : Pn;
-      const bool feas = wp.cfg.feasible;
+      const uint32_t v0 = s > base ? (uint32_t)(s - base) : 0u;
+      const uint32_t v1 = e - base < (u64)Pn ? (uint32_t)(e - base) : Pn;
+      // group tuples of the partition: table lookups (lane = (group, level))
+      bool infeas = false;
+      if (lane < k * L) {
+        const int b = lane / L, mu = lane % L;
+        const GroupRec r = gtab[(size_t)wp.cfg.mask[b] * L + mu];
+        wp.gt[b * L + mu] = r.t32;
+        wp.ge[b * L + mu] = r.e32;
+        wp.g64[b * L + mu] = r.t64;
+        infeas = r.t32 == __int_as_float(0x7f800000);
+      }
+      const bool feas = __ballot_sync(0xffffffffu, infeas) == 0u;
       if (lane == 0) {
         ncfg += v1 - v0;
         if (feas) nfeas += v1 - v0;
       }
-      if (feas) {
-        if (lane < k * L) {
-          const int b = lane / L, mu = lane % L;
-          float t32, e32;
-          double t64;
-          group_eval(tb, p, wp.cfg.mask[b], mu, t32, e32, t64);
-          wp.gt[b * L + mu] = t32;
-          wp.ge[b * L + mu] = e32;
-          wp.g64[b * L + mu] = t64;
-        }
-        __syncwarp();
-        nref += partition_configs<WS>(tb, p, stair, wp, thr, lb, v0, v1, lane);
-      }
+      __syncwarp();
+      if (feas) nref += partition_configs<WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
       __syncwarp();
       if (base + Pn >= e) break;
       if (lane == 0) {
@@ -461,7 +449,6 @@ __global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
         dev_successor(tb, p, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
-        cfg_feasibility(tb, p, wp.cfg);
       }
       __syncwarp();
     }
@@ -476,16 +463,17 @@ __global__ void __launch_bounds__(kTileThreads, 3) k_tile(const DevParams p) {
     }
   }
   // ---- reductions ----
+  u64 nref64 = (u64)nref;
 #pragma unroll
   for (int o = 16; o; o >>= 1) {
     ncfg += __shfl_xor_sync(0xffffffffu, ncfg, o);
     nfeas += __shfl_xor_sync(0xffffffffu, nfeas, o);
-    nref += __shfl_xor_sync(0xffffffffu, nref, o);
+    nref64 += __shfl_xor_sync(0xffffffffu, nref64, o);
   }
   if (lane == 0) {
     atomicAdd(p.ctr + kCtrConfigs, ncfg);
     atomicAdd(p.ctr + kCtrFeasible, nfeas);
-    atomicAdd(p.ctr + kCtrRefined, nref);
+    atomicAdd(p.ctr + kCtrRefined, nref64);
   }
 #pragma unroll
   for (int w = 0; w < WS::N; w++) {

@@ -40,11 +40,11 @@ static const void *tile_pick_ws(DevParams *dp) {
 
 size_t tile_smem_bytes(const DevParams &dp) {
   return ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(WarpPart) * kTileWarps +
-         sizeof(BestRec) * kTileWarps * kMaxW;
+         sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * kMaxW;
 }
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
-  if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4) return false;
+  if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4 || !dp.gtab_ok) return false;
   const void *fn = tile_pick_ws<4>(&dp);
   if (!fn) return false;
   tl->fn = fn;
