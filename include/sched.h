@@ -187,6 +187,21 @@ int sched_rank(const sched_query *q, const int8_t *group_of, const int8_t *level
 int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int32_t w,
                 sched_pick *out);
 
+/* The paper's rule-based co-scheduling heuristic (reading
+ * R25 in DESIGN.md), for measuring its optimality gap against the exhaustive
+ * search: (1) workflows in ascending solo SM utilisation (at 100 %), (2) a
+ * GPU's combined SM utilisation kept <= 100 %, (3) combined max memory <=
+ * capacity, (4) at most 2 clients per GPU if priority = throughput (0), at
+ * most max_clients if priority = energy (1).  Each workflow goes to the
+ * first open GPU satisfying (2)-(4), else a new GPU, else the open GPU with
+ * the lowest utilisation satisfying (3)-(4).  All clients run at the
+ * highest searched level.  Writes the configuration (canonical RGS,
+ * group_of/level_of as sched_unrank), its index in the query's space, and
+ * its fp64 score for weight w (out->valid = 0 if infeasible).  Host only.
+ * SCHED_E_INFEASIBLE if the rules cannot place every workflow. */
+int sched_heuristic(const sched_handle *h, const sched_query *q, int32_t priority, int32_t w,
+                    int8_t *group_of, int8_t *level_of, uint64_t *index, sched_pick *out);
+
 const char *sched_strerror(int status);
 
 /* Library version string, e.g. "sched-b200 0.1 sm_100a". */

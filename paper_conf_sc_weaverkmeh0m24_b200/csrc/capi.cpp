@@ -3,6 +3,7 @@
 // No exception crosses the ABI (every entry point catches).
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstring>
 #include <new>
@@ -342,6 +343,78 @@ int sched_score(const sched_handle *hc, const sched_query *qin, uint64_t index, 
   double T, E, ts, es;
   host_constants(h->P, q, &ts, &es);
   if (!host_score(h->P, q, a, k, dig, &T, &E)) return SCHED_OK;  // valid = 0: infeasible
+  out->valid = 1;
+  out->makespan_s = T;
+  out->energy_j = E;
+  out->x64 = ts / T;
+  out->y64 = es / E;
+  const int ea = q.nw ? q.wa[w] : 1, eb = q.nw ? q.wb[w] : 0;
+  out->score64 = host_objective(ts, es, T, E, ea, eb);
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_heuristic(const sched_handle *hc, const sched_query *qin, int32_t priority, int32_t w,
+                    int8_t *group_of, int8_t *level_of, uint64_t *index, sched_pick *out) {
+  GUARD_BEGIN
+  if (!hc || !group_of || !level_of || !index || !out || (priority != 0 && priority != 1))
+    return SCHED_E_INVALID;
+  sched_handle *h = const_cast<sched_handle *>(hc);
+  Query q;
+  const Space *sp;
+  int st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  if (w < 0 || (q.nw > 0 && w >= q.nw) || (q.nw == 0 && w != 0)) return SCHED_E_INVALID;
+  const Profile &P = h->P;
+  const int n = q.n, top = q.L - 1, lvl = q.lev[top];
+  // (1) ascending solo SM utilisation at 100 %, queue order on ties
+  int order[kMaxN];
+  for (int i = 0; i < n; i++) order[i] = i;
+  std::stable_sort(order, order + n, [&](int x, int y) {
+    return P.u[(size_t)x * P.lp + P.l100] < P.u[(size_t)y * P.lp + P.l100];
+  });
+  const int cap_clients = priority == 0 ? std::min(2, q.c) : q.c;
+  int gpu_of[kMaxN], ng = 0, cnt[kMaxG] = {0};
+  double util[kMaxG] = {0}, mem[kMaxG] = {0};
+  for (int r = 0; r < n; r++) {
+    const int i = order[r];
+    const double ui = P.u[(size_t)i * P.lp + lvl], mi = P.mem[i];
+    int pick = -1;
+    for (int g = 0; g < ng && pick < 0; g++)  // (2) (3) (4)
+      if (cnt[g] < cap_clients && util[g] + ui <= 1.0 && mem[g] + mi <= P.mem_cap) pick = g;
+    if (pick < 0 && ng < q.g) pick = ng++;
+    if (pick < 0) {  // no GPU keeps compute <= 100 %: least utilised one that fits (3) (4)
+      for (int g = 0; g < ng; g++)
+        if (cnt[g] < cap_clients && mem[g] + mi <= P.mem_cap && (pick < 0 || util[g] < util[pick])) pick = g;
+    }
+    if (pick < 0) return SCHED_E_INFEASIBLE;
+    gpu_of[i] = pick;
+    cnt[pick]++;
+    util[pick] += ui;
+    mem[pick] += mi;
+  }
+  // canonical RGS relabelling (groups by first member)
+  int relabel[kMaxG];
+  for (int g = 0; g < kMaxG; g++) relabel[g] = -1;
+  int k = 0;
+  int8_t a[kMaxN], dig[kMaxN];
+  for (int i = 0; i < n; i++) {
+    if (relabel[gpu_of[i]] < 0) relabel[gpu_of[i]] = k++;
+    a[i] = (int8_t)relabel[gpu_of[i]];
+  }
+  const int nd = q.scope == SCHED_PER_CLIENT ? n : k;
+  for (int d = 0; d < nd; d++) dig[d] = (int8_t)top;
+  st = host_rank(*sp, a, dig, index);
+  if (st) return st;
+  for (int i = 0; i < n; i++) {
+    group_of[i] = a[i];
+    level_of[i] = (int8_t)top;
+  }
+  std::memset(out, 0, sizeof *out);
+  out->index = *index;
+  double T, E, ts, es;
+  host_constants(P, q, &ts, &es);
+  if (!host_score(P, q, a, k, dig, &T, &E)) return SCHED_OK;
   out->valid = 1;
   out->makespan_s = T;
   out->energy_j = E;

@@ -251,12 +251,13 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
   for (int i = jb + 1; i < hi; i++) atomicMin(s.pm + i, vb);
 }
 
-// fp32 + exact fp64 makespan of group `m` with every member at level mu
+// fp32 tuple + exact canonical fp64 (T_g, E_g) of group `m` with every member
+// at level mu (canonical order of DESIGN.md section 2, as in refine64)
 __device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p, uint32_t m, int mu,
-                                           float &t32, float &e32, double &t64) {
+                                           float &t32, float &e32, double &t64, double &e64) {
   const int L = p.L;
   float U = 0.f, B = 0.f, D = 0.f;
-  double U64 = 0.0, B64 = 0.0;
+  double U64 = 0.0, B64 = 0.0, D64 = 0.0;
   for (uint32_t mm = m; mm; mm &= mm - 1) {
     const int r = (__ffs(mm) - 1) * L + mu;
     U += tb.u[r];
@@ -284,9 +285,14 @@ __device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p,
     const double tau = __dmul_rn(__dmul_rn((double)tb.traw[ri], s64), c);
     if (tau > Tg64) Tg64 = tau;
   }
+  for (uint32_t mm = m; mm; mm &= mm - 1) {
+    const int r = (__ffs(mm) - 1) * L + mu;
+    D64 = __dadd_rn(D64, __dmul_rn(__dsub_rn((double)tb.praw[r], p.ps), (double)tb.traw[r]));
+  }
   t32 = Tg;
   e32 = p.phat * Tg + D;
   t64 = Tg64;
+  e64 = __dadd_rn(__dmul_rn(p.ps, Tg64), D64);
 }
 
 // ------------------------------------------------------------ DP walk (RGS state)

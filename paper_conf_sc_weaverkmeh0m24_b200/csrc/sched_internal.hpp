@@ -118,9 +118,10 @@ struct BestRec {      // 48 B
   int valid, pad;
 };
 
-struct GroupRec {     // 16 B: one (group mask, level) tuple; t32 = +inf marks memory-infeasible
+struct GroupRec {     // 24 B: one (group mask, level) tuple; t32 = +inf marks memory-infeasible
   float t32, e32;     // normalised fp32 T_g / T_seq, E_g / E_seq of the hot loop
   double t64;         // exact canonical fp64 T_g
+  double e64;         // exact canonical fp64 E_g = P_s T_g + D_g
 };
 
 struct CandRec {      // 32 B

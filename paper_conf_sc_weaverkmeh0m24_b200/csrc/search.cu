@@ -238,10 +238,11 @@ __global__ void __launch_bounds__(256) k_groups(const DevParams p, GroupRec *gta
     r.t32 = __int_as_float(0x7f800000);
     r.e32 = 0.f;
     r.t64 = __longlong_as_double(0x7ff0000000000000ll);
+    r.e64 = 0.0;
     if (m != 0 && __popc(m) <= p.c) {
       long long M = 0;
       for (uint32_t mm = m; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
-      if (M <= (long long)p.mem_cap) group_eval(tb, p, m, mu, r.t32, r.e32, r.t64);
+      if (M <= (long long)p.mem_cap) group_eval(tb, p, m, mu, r.t32, r.e32, r.t64, r.e64);
     }
     gtab[id] = r;
   }

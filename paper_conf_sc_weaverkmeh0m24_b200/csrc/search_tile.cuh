@@ -88,6 +88,7 @@ struct WarpPart {
   u64 base;
   float gt[kTileMaxG * 4], ge[kTileMaxG * 4];
   double g64[kTileMaxG * 4];
+  double ge64[kTileMaxG * 4];  // exact canonical fp64 E_g per (group, level)
   float2 lp[64];  // loop-prefix (max T, sum E) over groups 0..k-6, one entry per digit string
 };
 
@@ -130,10 +131,11 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
   }
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
-  int lam[kMaxN];
-  for (int i = 0; i < p.n; i++) lam[i] = dig[wp.cfg.a[i]];
-  double T64r, E64;
-  refine64(tb, p, wp.cfg.mask, wp.cfg.k, lam, &T64r, &E64);
+  // fp64 canonical re-score from the exact group tuples: T = max_g T_g (exact),
+  // E = ((0 + E_0) + E_1) + ... in block order (the canonical order)
+  const double T64r = T64;
+  double E64 = 0.0;
+  for (int b = 0; b < wp.cfg.k; b++) E64 = __dadd_rn(E64, wp.ge64[b * 4 + dig[b]]);
   if constexpr (WS::N > 0) {
 #pragma unroll
     for (int s = 0; s < WS::N; s++) {
@@ -433,6 +435,7 @@ __global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
         wp.gt[b * L + mu] = r.t32;
         wp.ge[b * L + mu] = r.e32;
         wp.g64[b * L + mu] = r.t64;
+        wp.ge64[b * L + mu] = r.e64;
         infeas = r.t32 == __int_as_float(0x7f800000);
       }
       const bool feas = __ballot_sync(0xffffffffu, infeas) == 0u;

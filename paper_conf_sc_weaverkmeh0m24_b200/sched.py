@@ -28,7 +28,7 @@ PER_GPU = 1
 UINT64_MAX = (1 << 64) - 1
 
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
-           "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score",
+           "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score", "sched_heuristic",
            "sched_strerror", "sched_version"]
 
 
@@ -206,6 +206,18 @@ class Scheduler:
         npv = min(npar.value, pareto_cap) if q.want_pareto else 0
         return SearchResult(rc, [best[w] for w in range(nw)], [par[k] for k in range(npv)],
                             stats.as_dict())
+
+    def heuristic(self, q, priority="throughput", w=0):
+        """The paper's rule-based scheduler (criteria 1-4).
+        Returns (group_of, level_of, index, Pick)."""
+        a = (C.c_int8 * 32)()
+        lv = (C.c_int8 * 32)()
+        idx = C.c_uint64()
+        out = Pick()
+        pr = {"throughput": 0, "energy": 1}[priority]
+        _check(lib().sched_heuristic(self._h, C.byref(self.cquery(q)), pr, w, a, lv, C.byref(idx), C.byref(out)),
+               "sched_heuristic")
+        return [a[i] for i in range(q.n)], [lv[i] for i in range(q.n)], idx.value, out
 
     def score(self, q, index, w=0) -> Pick:
         out = Pick()

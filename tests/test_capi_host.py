@@ -146,3 +146,30 @@ def test_merge_host():
         front[(t, e)] = min(i, front.get((t, e), i))
     exp = sorted([(t, e, i) for (t, e), i in front.items()])
     assert [(p.makespan_s, p.energy_j, p.index) for p in par] == exp
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_heuristic_rules_and_gap(seed):
+    """The paper's rule-based scheduler: its configuration
+    obeys criteria 2-4 where possible, round-trips through rank/unrank, is
+    scored exactly like the oracle, and never beats the exhaustive optimum."""
+    n, g = 7, 4
+    prof = make_profile(n, levels=(50, 100), seed=60 + seed)
+    q = Query(n, g, n, (50, 100), PER_GPU, ((1, 1), (1, 0), (0, 1)), True)
+    sch = S.Scheduler(prof)
+    ref = oracle.search(prof, q)
+    for pr, lim in (("throughput", 2), ("energy", n)):
+        try:
+            a, lv, idx, pick = sch.heuristic(q, pr, 0)
+        except S.SchedError as e:
+            assert e.status == S.sched.SCHED_E_INFEASIBLE
+            continue
+        oa, od = oracle.config(q, idx)
+        assert oa == a
+        assert all(x == 1 for x in lv)                      # highest searched level (100 %)
+        assert max(a.count(b) for b in set(a)) <= lim      # criterion 4
+        for b in set(a):                                    # criterion 3
+            assert sum(int(prof.max_mem_mib[i]) for i in range(n) if a[i] == b) <= prof.mem_capacity_mib
+        ok, T, E = oracle.score(prof, q, oa, od)
+        assert pick.valid == ok and pick.makespan_s == T and pick.energy_j == E
+        assert pick.score64 <= ref["best"][0][1]
