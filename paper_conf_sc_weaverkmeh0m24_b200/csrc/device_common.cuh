@@ -228,7 +228,12 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
   const float val = __double2float_ru(__dmul_ru(__ddiv_ru(E, p.eseq), g1));
   const unsigned int vb = __float_as_uint(val);
   const int jb = bucket_of(T, p.bucket_base);
-  if (vb < __ldcg(p.stv + jb)) atomicMin(p.stv + jb, vb);
+  bool improved = false;
+  if (vb < __ldcg(p.stv + jb)) {
+    atomicMin(p.stv + jb, vb);
+    improved = true;
+  }
+  unsigned long long pr = ((unsigned long long)vb << 32) | 0xffffffffull;  // val-only entry
   if (slot < p.cand_cap) {
     CandRec *c = (CandRec *)p.cand + slot;
     c->idx = idx;
@@ -237,18 +242,68 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
     c->t32 = t32;
     c->e32 = e32;
     __threadfence();  // the record is visible before its slot is published
-    const unsigned long long pr = ((unsigned long long)vb << 32) | slot;
+    pr = ((unsigned long long)vb << 32) | slot;
     if (pr < __ldcg(p.stp + jb)) {
       atomicMin(p.stp + jb, pr);
-      atomicAdd(p.ctr + kCtrStairVer, 1ull);
+      improved = true;
     }
     atomicMin(s.bp + jb, pr);
   } else {
     atomicExch(p.ctr + kCtrOverflow, 1ull);
-    atomicAdd(p.ctr + kCtrStairVer, 1ull);
+  }
+  if (improved) {  // publish in the insertion log (seq = version)
+    const unsigned long long seq = atomicAdd(p.ctr + kCtrStairVer, 1ull);
+    LogEnt *L = (LogEnt *)p.stlog + (seq % kLog);
+    L->pr = pr;
+    L->jb = (unsigned int)jb;
+    __threadfence();
+    atomicExch(&L->tag, (unsigned int)(seq + 1));
   }
   const int hi = jb + 64 < kBuckets ? jb + 64 : kBuckets;
   for (int i = jb + 1; i < hi; i++) atomicMin(s.pm + i, vb);
+}
+
+// Bring this warp's view of the CTA staircase up to date with the global
+// insertion log (entries pos .. version-1); falls back to a full merge when
+// the ring buffer has wrapped.  Idempotent (monotone minima).  All lanes call.
+__device__ __forceinline__ void stair_sync(Stair s, const DevParams &p, u64 &pos, u64 ver) {
+  ver = __shfl_sync(0xffffffffu, ver, 0);  // one view of the version for the whole warp
+  if (ver == pos) return;
+  if (ver - pos > (u64)kLog) {
+    stair_merge(s, p);
+    pos = ver;
+    return;
+  }
+  const int lane = threadIdx.x & 31;
+  for (u64 q = pos; q < ver; q++) {
+    // lane 0 reads the entry (acquire on its tag) and broadcasts it: every
+    // lane must take the same branch (the ballots below need the full warp)
+    unsigned int tag = 0, jb = 0;
+    unsigned long long pr = 0;
+    if (lane == 0) {
+      const LogEnt *L = (const LogEnt *)p.stlog + (q % kLog);
+      asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(tag) : "l"(&L->tag) : "memory");
+      pr = __ldcg(&L->pr);
+      jb = __ldcg(&L->jb);
+    }
+    tag = __shfl_sync(0xffffffffu, tag, 0);
+    if (tag != (unsigned int)(q + 1)) {  // not yet visible: stop here
+      pos = q;
+      return;
+    }
+    pr = __shfl_sync(0xffffffffu, pr, 0);
+    jb = __shfl_sync(0xffffffffu, jb, 0);
+    const unsigned int vb = (unsigned int)(pr >> 32);
+    if (lane == 0 && (unsigned int)pr != 0xffffffffu && pr < s.bp[jb]) atomicMin(s.bp + jb, pr);
+    for (int i0 = (int)jb + 1; i0 < kBuckets; i0 += 32) {  // pm is non-increasing: stop at the first pm <= val
+      const int i = i0 + lane;
+      const bool need = i < kBuckets && s.pm[i] > vb;
+      if (need) atomicMin(s.pm + i, vb);
+      if (__ballot_sync(0xffffffffu, need) != 0xffffffffu) break;
+    }
+  }
+  pos = ver;
+  __syncwarp();
 }
 
 // fp32 tuple + exact canonical fp64 (T_g, E_g) of group `m` with every member

@@ -19,7 +19,8 @@ constexpr int kMaxW = SCHED_MAX_WEIGHTS;        // 8
 constexpr int kBuckets = 2048;                  // Pareto staircase buckets (per CTA)
 constexpr int kBucketShift = 45;                // of the fp64 bits of T: 128 buckets per binade
 constexpr uint16_t kNoState = 0xFFFF;
-constexpr int kUnitLog2 = 11;                   // generic kernel: 2048 configs per warp unit
+constexpr int kUnitLog2 = 11;
+constexpr int kLog = 4096;                      // staircase insertion log (ring buffer entries)                   // generic kernel: 2048 configs per warp unit
 
 // Validated host copy of sched_profile.
 struct Profile {
@@ -89,6 +90,7 @@ struct DevParams {
   unsigned int *thr;           // [kMaxW] global fp32 proxy threshold bits (min)
   unsigned int *stv;           // [kBuckets] min val of verified points per bucket
   unsigned long long *stp;     // [kBuckets] min (val << 32 | candidate slot) per bucket
+  unsigned char *stlog;        // [kLog] LogEnt: insertion log (seq = ctr[kCtrStairVer])
   unsigned char *slots;        // [grid][W] BestRec
   unsigned char *cand;         // [cand_cap] CandRec
   uint32_t cand_cap;
@@ -122,6 +124,11 @@ struct GroupRec {     // 24 B: one (group mask, level) tuple; t32 = +inf marks m
   float t32, e32;     // normalised fp32 T_g / T_seq, E_g / E_seq of the hot loop
   double t64;         // exact canonical fp64 T_g
   double e64;         // exact canonical fp64 E_g = P_s T_g + D_g
+};
+
+struct LogEnt {       // 16 B staircase insertion: bucket, (val << 32 | slot or 0xffffffff), tag = seq + 1
+  unsigned long long pr;
+  unsigned int jb, tag;
 };
 
 struct CandRec {      // 32 B

@@ -112,11 +112,7 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
     for (int w = 0; w < kMaxW; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
     if (p.want_pareto) {
-      const u64 v = __ldcg(p.ctr + kCtrStairVer);
-      if (v != stair_ver) {
-        stair_ver = v;
-        stair_merge(stair, p);
-      }
+      stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     }
 
     // lanes interleave (idx = s + lane + 32 j) or take contiguous runs
@@ -257,6 +253,9 @@ __global__ void k_init(const DevParams p, int keep) {
   const bool kept = keep && (t == kCtrStairVer || t == kCtrPass ||
                              (keep == 2 && (t == kCtrCand || t == kCtrOverflow)));
   if (t < kCtrN && !kept) p.ctr[t] = 0ull;
+  if (keep != 2)  // a fresh log (re-run: its slot ids are rewritten by k_reseed)
+    for (int i = t; i < kLog; i += blockDim.x) ((LogEnt *)p.stlog)[i].tag = 0u;
+  if (keep == 1 && t == kCtrStairVer) p.ctr[t] = (unsigned long long)kLog + 1;  // forces a full merge
   if (keep) return;
   if (t < kMaxW) p.thr[t] = 0x7f800000u;
   for (int i = t; i < kBuckets; i += blockDim.x) {
@@ -400,7 +399,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, blob, slots, cand, surv, keep, out, gtab, total;
+  size_t ctr, thr, stv, stp, stlog, blob, slots, cand, surv, keep, out, gtab, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -416,6 +415,7 @@ WsLayout layout(const DevParams &dp) {
   L.thr = take(4 * kMaxW);
   L.stv = take(4 * kBuckets);
   L.stp = take(8 * kBuckets);
+  L.stlog = take(sizeof(LogEnt) * kLog);
   L.blob = take(dp.blob_bytes);
   L.slots = take(sizeof(BestRec) * kMaxW * (size_t)kMaxGrid);
   L.cand = take(sizeof(CandRec) * (size_t)dp.cand_cap);
@@ -461,6 +461,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.thr = (unsigned int *)(ws + L.thr);
   dp.stv = (unsigned int *)(ws + L.stv);
   dp.stp = (unsigned long long *)(ws + L.stp);
+  dp.stlog = ws + L.stlog;
   dp.slots = ws + L.slots;
   dp.cand = ws + L.cand;
   dp.out = ws + L.out;

@@ -248,11 +248,7 @@ __global__ void __launch_bounds__(kDfsThreads, 2) k_dfs(const DevParams p) {
 #pragma unroll
     for (int q = 0; q < WS::N; q++) thr.v[q] = fminf(thr.v[q], __uint_as_float(__ldcg(p.thr + p.ws_perm[q])));
     if (p.want_pareto) {
-      const u64 v = __ldcg(p.ctr + kCtrStairVer);
-      if (v != stair_ver) {
-        stair_ver = v;
-        stair_merge(stair, p);
-      }
+      stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     }
     if (lane == 0) {  // unrank s, detach the last two workflows: prefix + completion ordinal
       dev_unrank(tb, p, s, w.cfg);
@@ -278,14 +274,11 @@ __global__ void __launch_bounds__(kDfsThreads, 2) k_dfs(const DevParams p) {
       w.base = s - ord;
     }
     __syncwarp();
-    u64 ver_pref = p.want_pareto ? __ldcg(p.ctr + kCtrStairVer) : 0;
+    u64 ver_pref = p.want_pareto ? __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0) : 0;
     for (;;) {
       if (p.want_pareto) {
-        if (ver_pref != stair_ver) {
-          stair_ver = ver_pref;
-          stair_merge(stair, p);
-        }
-        ver_pref = __ldcg(p.ctr + kCtrStairVer);
+        stair_sync(stair, p, stair_ver, ver_pref);
+        ver_pref = __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0);
       }
       const int k = w.cfg.k;
       // ---- per-prefix tables (lane-parallel) ----

@@ -402,25 +402,18 @@ __global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
 #pragma unroll
     for (int w = 0; w < WS::N; w++) thr.v[w] = fminf(thr.v[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
     if (p.want_pareto) {
-      const u64 v = __ldcg(p.ctr + kCtrStairVer);
-      if (v != stair_ver) {
-        stair_ver = v;
-        stair_merge(stair, p);
-      }
+      stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     }
     if (lane == 0) {
       dev_unrank(tb, p, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
-    u64 ver_pref = p.want_pareto ? __ldcg(p.ctr + kCtrStairVer) : 0;
+    u64 ver_pref = p.want_pareto ? __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0) : 0;
     for (;;) {
       if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
-        if (ver_pref != stair_ver) {
-          stair_ver = ver_pref;
-          stair_merge(stair, p);
-        }
-        ver_pref = __ldcg(p.ctr + kCtrStairVer);
+        stair_sync(stair, p, stair_ver, ver_pref);
+        ver_pref = __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0);
       }
       const u64 base = wp.base;
       const uint32_t Pn = (uint32_t)wp.cfg.Pn;

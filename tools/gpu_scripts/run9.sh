@@ -1,5 +1,5 @@
 echo "start $(date +%s)"
-timeout 1200 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -3
 echo "tests done $(date +%s)"
 timeout 600 python - <<'PY'
 import paper_conf_sc_weaverkmeh0m24_b200 as S
