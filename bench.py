@@ -175,9 +175,16 @@ def run_ours(args):
 
     rank, world, local = env()
     assert torch.cuda.is_available(), "bench.py needs a CUDA device"
+    # BENCH_SHARE_GPU=1 (tests only): every rank uses cuda:0 with a gloo group,
+    # to exercise the N > 1 path on a one-GPU box; NCCL otherwise.
+    share = os.environ.get("BENCH_SHARE_GPU") == "1"
+    local = 0 if share else local
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     prof, q = config(args.workload)
     nw = len(q.weights)
     space = S.count(q)
@@ -229,8 +236,9 @@ def run_ours(args):
     barrier()
     clk = clocks.stop()
     elapsed = ev0.elapsed_time(ev1)
+    rdev = "cpu" if share else "cuda"
     if world > 1:
-        t = torch.tensor([elapsed, float(ncfg)], dtype=torch.float64, device="cuda")
+        t = torch.tensor([elapsed, float(ncfg)], dtype=torch.float64, device=rdev)
         mx = t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
         dist.all_reduce(t, op=dist.ReduceOp.SUM)
@@ -256,7 +264,7 @@ def run_ours(args):
     barrier()
     e_dt = time.perf_counter() - t0
     if world > 1:
-        t = torch.tensor([e_dt, float(e_cfg)], dtype=torch.float64, device="cuda")
+        t = torch.tensor([e_dt, float(e_cfg)], dtype=torch.float64, device=rdev)
         mx = t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
         dist.all_reduce(t, op=dist.ReduceOp.SUM)
