@@ -100,7 +100,7 @@ typedef struct {
   uint64_t index_lo, index_hi;  /* searched window [lo, hi); hi = UINT64_MAX means |Omega| */
   int32_t shard_rank;           /* this rank's share: chunks c with c % shard_count == rank */
   int32_t shard_count;          /* >= 1 (multi-GPU split, one process per GPU) */
-  int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 10..40 (default 22) */
+  int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 12..40 (0 = default 22) */
   int32_t want_pareto;          /* nonzero: also compute the (T, E) Pareto set */
   uint32_t candidate_cap;       /* device Pareto-candidate buffer records; 0 = 1<<20 */
 } sched_query;
@@ -124,7 +124,7 @@ typedef struct {
   double t_seq_s, e_seq_j;      /* sequential baselines */
   float search_ms;              /* device time of the search kernel(s) (CUDA events) */
   float total_ms;               /* device time of the whole call on the stream */
-  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile kernel, 2 partition DFS kernel */
+  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile kernel, 2 L=1 pair kernel, 3 L=1 suffix kernel */
   int32_t grid_ctas;            /* persistent CTAs launched by the search kernel */
   int32_t kernel_launches;      /* kernels this call launched (init, search pass(es), finalize) */
   int32_t passes;               /* search passes (2 = re-run after candidate overflow) */

@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "device_common.cuh"
@@ -395,6 +396,15 @@ __global__ void k_pareto_order(const DevParams p, const unsigned int *surv, cons
 
 // ------------------------------------------------------------ launcher
 namespace {
+// SCHED_KERNEL=generic|tile|dfs|sfx restricts the kernel choice (testing and
+// measurement of the individual paths); unset = the fastest eligible path.
+bool want_path(int path) {
+  static const char *names[] = {"generic", "tile", "dfs", "sfx"};
+  const char *e = std::getenv("SCHED_KERNEL");
+  if (!e || !*e) return true;
+  return std::strcmp(e, names[path]) == 0;
+}
+
 constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
@@ -520,10 +530,13 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       launches++;
     }
     TileLaunch tl;
-    if (tile_eligible(dp, &tl)) {
+    if (want_path(1) && tile_eligible(dp, &tl)) {
       path = 1;
       CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
-    } else if (dfs_eligible(dp, &tl)) {
+    } else if (want_path(3) && sfx_eligible(dp, &tl)) {
+      path = 3;
+      CK(launch_sfx(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
+    } else if (want_path(2) && dfs_eligible(dp, &tl)) {
       path = 2;
       CK(launch_dfs(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
     } else {

@@ -1,0 +1,48 @@
+// sfx_host.cu -- eligibility and launch of the L = 1 suffix kernel
+// (search_sfx.cuh); instantiations in sfx_<M>.cu.
+#include "search_sfx.cuh"
+
+namespace sched {
+
+static size_t sfx_smem(const DevParams &dp, int M) {
+  const size_t warp = M == 6 ? sizeof(SfxWarp<6>) : sizeof(SfxWarp<4>);
+  return ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + warp * kSfxWarps + sizeof(BestRec) * kSfxWarps * kMaxW;
+}
+
+bool sfx_eligible(DevParams &dp, TileLaunch *tl) {
+  if (dp.L != 1 || dp.g > kSfxMaxG || (dp.capped && dp.c > 15) || !dp.gtab_ok) return false;
+  int M;
+  if (dp.n >= 8) M = 6;
+  else if (dp.n >= 6) M = 4;
+  else return false;
+  tl->fn = M == 6 ? sfx_fn<6>() : sfx_fn<4>();
+  tl->smem = sfx_smem(dp, M);
+  return true;
+}
+
+cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                       cudaEvent_t e2, int *grid, bool fixed_units) {
+  cudaError_t err = cudaFuncSetAttribute(tl.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tl.smem);
+  if (err != cudaSuccess) return err;
+  int occ = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kSfxThreads, tl.smem);
+  if (err != cudaSuccess) return err;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  *grid = std::min(4096, nsm * occ);
+  if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
+    const uint64_t range = dp.n_owned << dp.chunk_log2;
+    const uint64_t warps = (uint64_t)(*grid) * kSfxWarps;
+    int ul = 12;
+    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 8) ul++;
+    dp.unit_log2 = ul;
+    dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+    dp.unit_stride = 1;
+  }
+  void *args[] = {(void *)&dp};
+  cudaEventRecord(e1, st);
+  err = cudaLaunchKernel(tl.fn, *grid, kSfxThreads, args, tl.smem, st);
+  cudaEventRecord(e2, st);
+  return err;
+}
+
+}  // namespace sched

@@ -203,9 +203,10 @@ def test_full_space_vs_dp_certificate(name):
     (9, 4, 3, ((1, 0), (3, 1), (2, 1), (1, 1), (1, 2), (1, 3), (0, 1)), 1),
     (10, 5, 2, ((1, 1),), 2), (8, 8, 4, ((1, 1), (2, 1)), 3), (11, 4, 3, (), 4), (7, 3, 4, ((1, 0),), 5),
 ])
-def test_partition_kernel_path(n, g, c, ws, seed):
-    """L = 1 spaces (every configuration is a partition) run on the partition
-    kernel (kernel_path 2) and must equal the oracle exactly."""
+def test_partition_kernel_path(n, g, c, ws, seed, monkeypatch):
+    """L = 1 spaces (every configuration is a partition) on the pair kernel
+    (kernel_path 2, SCHED_KERNEL=dfs) must equal the oracle exactly."""
+    monkeypatch.setenv("SCHED_KERNEL", "dfs")
     prof = make_profile(n, levels=(100,), seed=seed)
     q = Query(n, g, c, (100,), PER_GPU, ws, True)
     res = S.Scheduler(prof).search(q)
