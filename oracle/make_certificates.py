@@ -13,7 +13,7 @@ GOLD = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
 
 
 def main():
-    for name in ("c3", "c4"):
+    for name in ("c3", "c4", "c5"):
         prof, q = config(name)
         c = oracle.dp_certificate(prof, q)
         out = {"config": name, "source": "oracle.dp_certificate (oracle/dpcert.c, O3), seed 0 synth.config",

@@ -181,9 +181,9 @@ def _certificate(name):
     return front, best
 
 
-@pytest.mark.parametrize("name", ["c3", "c4"])
+@pytest.mark.parametrize("name", ["c3", "c4", "c5"])
 def test_full_space_vs_dp_certificate(name):
-    """Full c3 / c4 search (c4: 2.07e14 configurations, ~70 s on one B200) in
+    """Full c3 / c4 / c5 search (c4: 2.07e14 configurations, ~60 s on one B200) in
     the bench's launch configuration vs the O3 subset-DP certificate
     (tests/golden/<cfg>_certificate.json, written by oracle/make_certificates.py):
     the Pareto front values and the optimum of every weight must be bitwise

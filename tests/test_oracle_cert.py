@@ -1,6 +1,6 @@
 """O3 (subset-DP certificate) pinned against O1 (full enumeration) on every
 PER_GPU space small enough to enumerate: Pareto-front values and the
-optimum of every weight must be bitwise equal.  The stored c3/c4
+optimum of every weight must be bitwise equal.  The stored c3/c4/c5
 certificates (tests/golden) must be reproducible from oracle/ alone."""
 import json
 import os
@@ -16,7 +16,7 @@ W = ((1, 1), (2, 1), (1, 0), (0, 1), (1, 3))
 @pytest.mark.parametrize("n,g,c,levels,seed", [
     (5, 2, 3, (50, 100), 1), (6, 3, 3, (25, 50, 100), 2), (7, 4, 7, (50, 100), 3),
     (8, 3, 3, (25, 50, 75, 100), 4), (9, 4, 4, (50, 100), 5), (8, 8, 8, (100,), 6),
-    (9, 5, 2, (25, 100), 7),
+    (9, 5, 2, (25, 100), 7), (10, 4, 3, (100,), 9),   # last: the c5 shape (L = 1, C = 3)
 ])
 def test_certificate_equals_enumeration(n, g, c, levels, seed):
     prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
@@ -36,7 +36,7 @@ def test_certificate_handles_infeasible_groups():
     assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
 
 
-@pytest.mark.parametrize("name", ["c3", "c4"])
+@pytest.mark.parametrize("name", ["c3", "c4", "c5"])
 def test_golden_certificates_reproduce(name):
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"{name}_certificate.json")))
     prof, q = config(name)
