@@ -86,15 +86,14 @@ __device__ __forceinline__ uint32_t sfx_opts(const SfxLane &s, int G) {
 __device__ __forceinline__ void sfx_apply(SfxLane &s, int j, uint32_t bi, float2 v, int C) {
   s.T = fmaxf(s.T, v.x);
   s.E = s.E + v.y;
-  if (j == s.kc) {
-    s.kc++;
-    const uint32_t room = (uint32_t)(C - 1 < 15 ? C - 1 : 15);
-    s.rr |= room << (4 * j);
-    if (room) s.rm |= 1u << j;
-  } else {
-    s.rr -= 1u << (4 * j);
-    if (((s.rr >> (4 * j)) & 15u) == 0u) s.rm &= ~(1u << j);
-  }
+  // branchless: a new group (j == kc) gets room min(C-1, 15) in its (zero)
+  // nibble, an existing one loses one unit of room
+  const bool nw = j == s.kc;
+  const uint32_t room = (uint32_t)(C - 1 < 15 ? C - 1 : 15);
+  s.kc += nw ? 1 : 0;
+  s.rr += (nw ? room : 0xffffffffu) << (4 * j);
+  const uint32_t has = ((s.rr >> (4 * j)) & 15u) ? 1u : 0u;
+  s.rm = (s.rm & ~(1u << j)) | (has << j);
   s.gi |= (u64)bi << (8 * j);
 }
 
@@ -145,9 +144,56 @@ static __device__ __noinline__ void sfx_check(const DevParams &p, const Stair &s
     emit_candidate(p, stair, idx, T64, E64, T, E);
 }
 
-// Level I of the lexicographic enumeration (placement of suffix element I).
-// first: still on the first descent (start at the unranked choice start[I]).
-// CHECK = false: fast pass (T, E, min-reduce); true: per-configuration checks.
+// The last level (suffix element M-1) over the option set `opts` of state
+// st: every option is one configuration.  FAST: (T, E) and the lane's
+// min-reduction (the loop carries no count or order bookkeeping; options
+// are taken highest first); CHECK: ascending (lexicographic) order with the
+// exact ordinal, per-configuration screens.  lim bounds the number taken.
+template <int M, bool CHECK>
+__device__ __forceinline__ void sfx_last(const DevParams &p, const Stair &stair, const SfxCtx &x, SfxHot &h,
+                                         SfxCold *cold, const SfxLane &st, uint32_t opts) {
+  constexpr int RS = SfxWarp<M>::RS;
+  constexpr uint32_t bl = 1u << (M - 1);
+  if constexpr (!CHECK) {
+    float mT = h.mT, mE = h.mE;
+    int nf = h.nf;
+    while (opts) {
+      uint32_t j;
+      asm("bfind.u32 %0, %1;" : "=r"(j) : "r"(opts));
+      opts ^= 1u << j;
+      const float2 v = x.tab[j * RS + (((uint32_t)(st.gi >> (8 * j)) & 0xffu) | bl)];
+      const float T = fmaxf(st.T, v.x), E = st.E + v.y;
+      mT = fminf(mT, T);
+      mE = fminf(mE, E);
+      nf += (int)((__float_as_uint(T) - 0x7f800000u) >> 31);  // T < +inf (T >= 0)
+    }
+    h.mT = mT;
+    h.mE = mE;
+    h.nf = nf;
+  } else {
+    while (opts) {
+      const int j = __ffs(opts) - 1;
+      opts &= opts - 1;
+      const float2 v = x.tab[j * RS + (((uint32_t)(st.gi >> (8 * j)) & 0xffu) | bl)];
+      const float T = fmaxf(st.T, v.x), E = st.E + v.y;
+      const int kc = st.kc + (j == st.kc ? 1 : 0);
+      sfx_check(p, stair, x, cold, st.gi | ((u64)bl << (8 * j)), kc, T, E, x.base + h.ord);
+      h.ord++;
+    }
+  }
+}
+
+// m without its `lim` lowest set bits
+__device__ __forceinline__ uint32_t strip_low(uint32_t m, int lim) {
+  for (; lim > 0 && m; lim--) m &= m - 1;
+  return m;
+}
+
+// Level I < M-1 of the lexicographic enumeration (placement of suffix
+// element I).  first: still on the first descent (start at the unranked
+// choice start[I]).  h.cnt = configurations left in the lane's range; the
+// level above the last checks it once per option, so the last level runs
+// without bookkeeping.
 template <int M, int I, bool CHECK>
 __device__ __forceinline__ void sfx_level(const DevParams &p, const Stair &stair, const SfxCtx &x, SfxHot &h,
                                           SfxCold *cold, const SfxLane &st, bool first) {
@@ -159,26 +205,137 @@ __device__ __forceinline__ void sfx_level(const DevParams &p, const Stair &stair
     const int j = __ffs(opts) - 1;
     opts &= opts - 1;
     const float2 v = x.tab[j * RS + (((uint32_t)(st.gi >> (8 * j)) & 0xffu) | bi)];
-    if constexpr (I == M - 1) {
-      const float T = fmaxf(st.T, v.x), E = st.E + v.y;
-      if constexpr (!CHECK) {
-        h.mT = fminf(h.mT, T);
-        h.mE = fminf(h.mE, E);
-        h.nf += T < __int_as_float(0x7f800000) ? 1 : 0;
-      } else {
-        const int kc = st.kc + (j == st.kc ? 1 : 0);
-        sfx_check(p, stair, x, cold, st.gi | ((u64)bi << (8 * j)), kc, T, E, x.base + h.ord);
-        h.ord++;
+    SfxLane s2 = st;
+    sfx_apply(s2, j, bi, v, x.C);
+    if constexpr (I == M - 2) {
+      uint32_t o2 = sfx_opts(s2, x.G);
+      if (first) o2 &= ~0u << x.start[M - 1];
+      const int n2 = __popc(o2);
+      if (h.cnt > n2) {
+        sfx_last<M, CHECK>(p, stair, x, h, cold, s2, o2);
+        h.cnt -= n2;
+      } else {  // the lane's range ends inside this option set
+        sfx_last<M, CHECK>(p, stair, x, h, cold, s2, o2 & ~strip_low(o2, h.cnt));
+        h.cnt = 0;
+        return;
       }
-      if (--h.cnt == 0) return;
     } else {
-      SfxLane s2 = st;
-      sfx_apply(s2, j, bi, v, x.C);
       sfx_level<M, I + 1, CHECK>(p, stair, x, h, cold, s2, first);
       if (h.cnt == 0) return;
     }
     first = false;
   }
+}
+
+// ---- fast pass: converged per-parent loop ----
+// A parent is a state after x_0..x_{M-2}; its configurations are the options
+// of the last element.  sfx_slots evaluates them over the 8 row slots
+// without branches: a full group's entry (|S| > cap) is (+inf, +inf); rows
+// >= G hold (+inf, +inf); slots kc+1 .. G-1 are empty "new" rows whose entry
+// repeats the new-group configuration of slot kc (mins unchanged, the
+// feasible count is corrected).  Every lane runs the same instructions.
+template <int M>
+__device__ __forceinline__ void sfx_slots(const float2 *tab, const SfxLane &s, int G, float &mT, float &mE,
+                                          int &nf) {
+  constexpr int RS = SfxWarp<M>::RS;
+  constexpr uint32_t bl = 1u << (M - 1);
+  const uint32_t lo = (uint32_t)s.gi, hi = (uint32_t)(s.gi >> 32);
+  int c = 0;
+#pragma unroll
+  for (int j = 0; j < kSfxMaxG; j++) {
+    const uint32_t S = __byte_perm(j < 4 ? lo : hi, 0u, 0x4440u | (uint32_t)(j & 3));
+    const float2 v = tab[j * RS + bl + S];  // S | bl == S + bl
+    const float T = fmaxf(s.T, v.x), E = s.E + v.y;
+    mT = fminf(mT, T);
+    mE = fminf(mE, E);
+    c += (int)((__float_as_uint(T) - 0x7f800000u) >> 31);
+  }
+  if (s.kc < G - 1) {  // duplicates of the new-group configuration
+    const float T = fmaxf(s.T, tab[(G - 1) * RS + bl].x);
+    c -= (G - 1 - s.kc) * (int)((__float_as_uint(T) - 0x7f800000u) >> 31);
+  }
+  nf += c;
+}
+
+// next option at level I (I <= M-2) and the first parent below it; false
+// when level I is exhausted.  st[I] = state before x_I, rem[I] = options left.
+template <int M, int I>
+__device__ __forceinline__ bool sfx_adv(const SfxCtx &x, SfxLane (&st)[M - 1], uint32_t (&rem)[M - 1],
+                                        SfxLane &par) {
+  constexpr int RS = SfxWarp<M>::RS;
+  while (rem[I]) {
+    const int j = __ffs(rem[I]) - 1;
+    rem[I] &= rem[I] - 1;
+    const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
+    SfxLane s = st[I];
+    sfx_apply(s, j, 1u << I, v, x.C);
+    if constexpr (I == M - 2) {
+      par = s;
+      return true;
+    } else {
+      st[I + 1] = s;
+      rem[I + 1] = sfx_opts(s, x.G);
+      if (sfx_adv<M, I + 1>(x, st, rem, par)) return true;
+    }
+  }
+  return false;
+}
+
+template <int M, int I>
+__device__ __forceinline__ bool sfx_next(const SfxCtx &x, SfxLane (&st)[M - 1], uint32_t (&rem)[M - 1],
+                                         SfxLane &par) {
+  if (sfx_adv<M, I>(x, st, rem, par)) return true;
+  if constexpr (I == 0) {
+    return false;
+  } else {
+    return sfx_next<M, I - 1>(x, st, rem, par);
+  }
+}
+
+// Fast pass over the lane range starting at the unranked choices x.start
+// (state s0 before x_0), cnt configurations.
+template <int M>
+__device__ __forceinline__ void sfx_fast(const DevParams &p, const Stair &stair, const SfxCtx &x, SfxHot &h,
+                                         const SfxLane &s0, int cnt) {
+  constexpr int RS = SfxWarp<M>::RS;
+  SfxLane st[M - 1], par;
+  uint32_t rem[M - 1];
+  st[0] = s0;
+#pragma unroll
+  for (int I = 0; I < M - 1; I++) {
+    const int j = x.start[I];
+    rem[I] = sfx_opts(st[I], x.G) & (~1u << j);  // options after the start choice
+    const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
+    SfxLane s = st[I];
+    sfx_apply(s, j, 1u << I, v, x.C);
+    if (I < M - 2) st[I + 1] = s;
+    else par = s;
+  }
+  uint32_t o = sfx_opts(par, x.G) & (~0u << x.start[M - 1]);
+  for (;;) {
+    const int n = __popc(o);
+    if (cnt <= n) {  // the lane's range ends in this parent
+      sfx_last<M, false>(p, stair, x, h, nullptr, par, o & ~strip_low(o, cnt));
+      return;
+    }
+    if (o == sfx_opts(par, x.G)) sfx_slots<M>(x.tab, par, x.G, h.mT, h.mE, h.nf);
+    else sfx_last<M, false>(p, stair, x, h, nullptr, par, o);  // the partial first parent
+    cnt -= n;
+    if (!sfx_next<M, M - 2>(x, st, rem, par)) return;
+    o = sfx_opts(par, x.G);
+  }
+}
+
+// Slow pass over a lane range (out of line: keeps the fast pass's registers).
+template <int M>
+static __device__ __noinline__ void sfx_slow(const DevParams &p, const Stair &stair, const SfxCtx &x,
+                                             SfxCold *cold, const SfxLane &s0, uint32_t l0, int cnt) {
+  SfxHot h;
+  h.mT = h.mE = 0.f;
+  h.nf = 0;
+  h.cnt = cnt;
+  h.ord = l0;
+  sfx_level<M, 0, true>(p, stair, x, h, cold, s0, true);
 }
 
 // lane start: unrank ordinal r within the prefix's completions (DP table),
@@ -284,14 +441,16 @@ __device__ __forceinline__ bool sfx_prefix_successor(const Tables &tb, const Dev
 }
 
 // (t, de) of one table entry: group = key | S (suffix bits at `off`)
+// (values scaled by 1/T_seq, 1/E_seq: multiplication by a positive constant
+// is monotone, so T stays monotone along every chain; relative error <= 2u)
 __device__ __forceinline__ float2 sfx_entry(const DevParams &p, const GroupRec *gtab, uint32_t key, uint32_t S,
-                                            int off, int cap) {
+                                            int off, int cap, double its, double ies) {
   const float inf = __int_as_float(0x7f800000);
   if (S == 0u) {
     if (key == 0u) return make_float2(0.f, 0.f);
     const GroupRec g = gtab[key];
     if (!(g.t32 < inf)) return make_float2(inf, inf);
-    return make_float2(__double2float_rn(__ddiv_rn(g.t64, p.tseq)), __double2float_rn(__ddiv_rn(g.e64, p.eseq)));
+    return make_float2(__double2float_rn(__dmul_rn(g.t64, its)), __double2float_rn(__dmul_rn(g.e64, ies)));
   }
   if (__popc(S) > cap) return make_float2(inf, inf);
   const GroupRec cur = gtab[key | (S << off)];
@@ -299,8 +458,8 @@ __device__ __forceinline__ float2 sfx_entry(const DevParams &p, const GroupRec *
   const uint32_t Sp = S & ~(1u << (31 - __clz(S)));
   const uint32_t mp = key | (Sp << off);
   const double ep = mp ? gtab[mp].e64 : 0.0;
-  return make_float2(__double2float_rn(__ddiv_rn(cur.t64, p.tseq)),
-                     __double2float_rn(__ddiv_rn(__dsub_rn(cur.e64, ep), p.eseq)));
+  return make_float2(__double2float_rn(__dmul_rn(cur.t64, its)),
+                     __double2float_rn(__dmul_rn(__dsub_rn(cur.e64, ep), ies)));
 }
 
 template <int M>
@@ -317,11 +476,14 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
   BestRec *red = (BestRec *)(wps + kSfxWarps);
   stair_init(stair);
   if (lane < kSfxMaxG) w.key[lane] = 0xffffffffu;
+  for (int i = p.g * RS + lane; i < kSfxMaxG * RS; i += 32)  // rows >= G: no group
+    w.tab[i] = make_float2(__int_as_float(0x7f800000), __int_as_float(0x7f800000));
   __syncthreads();
 
   const GroupRec *gtab = (const GroupRec *)p.gtab;
   const int plen = p.n - M, off = p.n - M;
   const float inf = __int_as_float(0x7f800000);
+  const double its = 1.0 / p.tseq, ies = 1.0 / p.eseq;
   SfxCold cold;
 #pragma unroll
   for (int q = 0; q < kMaxW; q++) {
@@ -365,7 +527,7 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
         const uint32_t key = r < kp ? w.cfg.mask[r] : 0u;
         if (w.key[r] == key) continue;
         const int cap = key ? p.c - __popc(key) : p.c;
-        for (int S = lane; S < (1 << M); S += 32) w.tab[r * RS + S] = sfx_entry(p, gtab, key, (uint32_t)S, off, cap);
+        for (int S = lane; S < (1 << M); S += 32) w.tab[r * RS + S] = sfx_entry(p, gtab, key, (uint32_t)S, off, cap, its, ies);
         __syncwarp();
         if (lane == 0) w.key[r] = key;
       }
@@ -420,7 +582,7 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
           h.nf = 0;
           h.cnt = (int)(l1 - l0);
           h.ord = l0;
-          sfx_level<M, 0, false>(p, stair, x, h, &cold, s0, true);
+          sfx_fast<M>(p, stair, x, h, s0, (int)(l1 - l0));
           nfeas += (u64)h.nf;
           if (h.nf) {
             bool hit = false;
@@ -434,11 +596,7 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
               }
             }
             if (!hit && p.want_pareto) hit = !stair_dominated_f(stair, p, __fmul_rd(h.mT, p.tlb_scale_f), h.mE);
-            if (hit) {
-              h.cnt = (int)(l1 - l0);
-              h.ord = l0;
-              sfx_level<M, 0, true>(p, stair, x, h, &cold, s0, true);
-            }
+            if (hit) sfx_slow<M>(p, stair, x, &cold, s0, l0, (int)(l1 - l0));
           }
         }
       }
