@@ -53,7 +53,8 @@ class _Query(C.Structure):
     _fields_ = [("n", C.c_int), ("g", C.c_int), ("c", C.c_int), ("L", C.c_int),
                 ("lev", C.POINTER(C.c_int)), ("scope", C.c_int), ("nw", C.c_int),
                 ("wa", C.POINTER(C.c_int)), ("wb", C.POINTER(C.c_int)),
-                ("lo", C.c_uint64), ("hi", C.c_uint64), ("want_pareto", C.c_int)]
+                ("lo", C.c_uint64), ("hi", C.c_uint64), ("want_pareto", C.c_int),
+                ("model", C.c_uint), ("power_cap", C.c_float)]
 
 
 class _Best(C.Structure):
@@ -109,7 +110,8 @@ class _Pack:
         hi = q.index_hi if q.index_hi is not None else count(q)
         self.Q = _Query(q.n, q.g, min(q.c, q.n), len(q.levels), _ptr(lev, C.c_int),
                         q.scope, len(q.weights), _ptr(wa, C.c_int), _ptr(wb, C.c_int),
-                        int(q.index_lo), int(hi), int(bool(q.want_pareto)))
+                        int(q.index_lo), int(hi), int(bool(q.want_pareto)),
+                        int(getattr(q, "model", 0)), float(getattr(q, "power_cap", 0.0)))
 
 
 def count(q) -> int:
@@ -225,7 +227,7 @@ def score(prof, q, rgs, digits):
     plc = (C.c_int * 64)(*pl)
     T = C.c_double()
     E = C.c_double()
-    ok = lib().oracle_score_config(C.byref(pk.P), q.n, a, k, plc, C.byref(T), C.byref(E))
+    ok = lib().oracle_score_config(C.byref(pk.P), C.byref(pk.Q), q.n, a, k, plc, C.byref(T), C.byref(E))
     return bool(ok), T.value, E.value
 
 

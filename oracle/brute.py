@@ -35,22 +35,43 @@ def space(n, g, c, L, scope):
     return out
 
 
-def t_seq(t100, g):
+COUNT_IDLE, NO_INTERFERENCE, POWER_CAP = 1, 2, 4   # scoring-model variants (R26-R28)
+
+
+def _capped(t, dyn, capd):
+    """solo / group time under the power cap: max(t, dyn / (P_cap - P_s))"""
+    tc = dyn / capd
+    return tc if tc > t else t
+
+
+def t_seq(t100, g, p100=None, ps=0.0, model=0, pcap=0.0):
     fin = [0.0] * g
-    for ti in t100:
+    for i, ti in enumerate(t100):
+        if model & POWER_CAP:
+            ti = _capped(ti, (p100[i] - ps) * ti, pcap - ps)
         j = min(range(g), key=lambda x: (fin[x], x))
         fin[j] = fin[j] + ti
     return max(fin)
 
 
-def e_seq(p100, t100):
+def e_seq(p100, t100, ps=0.0, model=0, pcap=0.0, g=1, ts=0.0):
     e = 0.0
+    if model & COUNT_IDLE:
+        for pi, ti in zip(p100, t100):
+            e = e + (pi - ps) * ti
+        return (g * ps) * ts + e
     for pi, ti in zip(p100, t100):
-        e = e + pi * ti
+        ei = pi * ti
+        if model & POWER_CAP:
+            dyn = (pi - ps) * ti
+            tc = _capped(ti, dyn, pcap - ps)
+            if tc != ti:
+                ei = ps * tc + dyn
+        e = e + ei
     return e
 
 
-def score(prof, n, rgs, lv_prof):
+def score(prof, n, rgs, lv_prof, model=0, pcap=0.0, g=1):
     """lv_prof[i]: profile level index of workflow i. -> (feasible, T, E)."""
     t = prof.solo_time_s.astype(float)
     p = prof.solo_power_w.astype(float)
@@ -65,12 +86,15 @@ def score(prof, n, rgs, lv_prof):
             return False, None, None
     T = 0.0
     E = 0.0
+    Dall = 0.0
     for grp in groups:
         U = 0.0
         B = 0.0
         for i in grp:
             U = U + u[i, lv_prof[i]]
             B = B + bw[i, lv_prof[i]]
+        if model & NO_INTERFERENCE and (U > 1.0 or B > 1.0):
+            return False, None, None
         cg = max(max(1.0, U), B)
         Tg = 0.0
         for i in grp:
@@ -83,8 +107,13 @@ def score(prof, n, rgs, lv_prof):
         D = 0.0
         for i in grp:
             D = D + (p[i, lv_prof[i]] - ps) * t[i, lv_prof[i]]
+        if model & POWER_CAP:
+            Tg = _capped(Tg, D, float(pcap) - ps)
         T = max(T, Tg)
         E = E + (ps * Tg + D)
+        Dall = Dall + D
+    if model & COUNT_IDLE:
+        E = (g * ps) * T + Dall
     return True, T, E
 
 
@@ -94,14 +123,17 @@ def search(prof, q):
     l100 = pct.index(100)
     t100 = [float(prof.solo_time_s[i, l100]) for i in range(q.n)]
     p100 = [float(prof.solo_power_w[i, l100]) for i in range(q.n)]
-    ts = t_seq(t100, q.g)
-    es = e_seq(p100, t100)
+    model = getattr(q, "model", 0)
+    pcap = float(getattr(q, "power_cap", 0.0))
+    ps = float(prof.static_power_w)
+    ts = t_seq(t100, q.g, p100, ps, model, pcap)
+    es = e_seq(p100, t100, ps, model, pcap, q.g, ts)
     sp = space(q.n, q.g, min(q.c, q.n), len(q.levels), q.scope)
     best = [None] * len(q.weights)
     feas = []
     for idx, (rgs, dig) in enumerate(sp):
         lvp = [lev[dig[i]] if q.scope == PER_CLIENT else lev[dig[rgs[i]]] for i in range(q.n)]
-        ok, T, E = score(prof, q.n, rgs, lvp)
+        ok, T, E = score(prof, q.n, rgs, lvp, model, pcap, q.g)
         if not ok:
             continue
         feas.append((idx, T, E))

@@ -36,6 +36,25 @@
  *  Results: best index per weight (max F, ties -> lowest index) and the
  *  Pareto set of distinct (T,E) over feasible configurations, one (lowest)
  *  index per point.
+ *
+ *  Scoring-model variants (readings R26-R28 in DESIGN.md),
+ *  selected by or_query.model bits; 0 is the canonical model above:
+ *   1 COUNT_IDLE: every one of the G GPUs draws P_s for the whole makespan
+ *     (R8 variant).  With E_g = P_s*T_g + D_g this is
+ *       E = (G*P_s)*T + D,  D = sum_g D_g (group order),
+ *     and the sequential baseline likewise E_seq = (G*P_s)*T_seq + sum_i dyn_i.
+ *   2 NO_INTERFERENCE: the PAPER.md L87 predicate as a hard rule ("two
+ *     workflows are predicted to interfere if ... combined average SM
+ *     utilization over 100%, combined average memory bandwidth utilization
+ *     over 100%", criterion 2 "kept under 100%", L90): a group with
+ *     U_g > 1 or B_g > 1 is infeasible.
+ *   4 POWER_CAP: software power capping at P_cap (PAPER.md L162, 300 W on
+ *     A100X): a group whose average power P_s + D_g/T_g exceeds P_cap is
+ *     throttled until it does not, its dynamic energy conserved:
+ *       T_g' = max(T_g, D_g / (P_cap - P_s)),  E_g = P_s*T_g' + D_g.
+ *     A solo task in the sequential baseline likewise runs for
+ *     t' = max(t, dyn / (P_cap - P_s)); its energy stays p*t when not capped,
+ *     else P_s*t' + dyn.
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -60,7 +79,13 @@ typedef struct {
   const int *wa, *wb;      /* [nw] exponents */
   uint64_t lo, hi;         /* index window [lo, hi) */
   int want_pareto;
+  unsigned model;          /* variant bits: 1 COUNT_IDLE, 2 NO_INTERFERENCE, 4 POWER_CAP */
+  float power_cap;         /* P_cap (W) for POWER_CAP */
 } or_query;
+
+#define OR_COUNT_IDLE 1u
+#define OR_NO_INTERFERENCE 2u
+#define OR_POWER_CAP 4u
 
 typedef struct { uint64_t idx; double f, t, e; int found; } or_best;
 typedef struct { uint64_t idx; double t, e; } or_point;
@@ -139,25 +164,47 @@ void oracle_count(const or_query *q, uint64_t *lo, uint64_t *hi) {
 /* -------------------------------------------------------------- constants */
 void oracle_constants(const or_profile *P, const or_query *q, int l100,
                       double *tseq, double *eseq) {
+  const double ps = (double)P->ps;
+  const double capd = (double)q->power_cap - ps;   /* exact: two floats */
   double fin[64];
   for (int g = 0; g < q->g; g++) fin[g] = 0.0;
   for (int i = 0; i < q->n; i++) {          /* queue order, min finish, lowest id */
+    double t = (double)P->t[i * P->lp + l100];
+    if (q->model & OR_POWER_CAP) {
+      double tc = (((double)P->p[i * P->lp + l100] - ps) * t) / capd;
+      if (tc > t) t = tc;
+    }
     int best = 0;
     for (int g = 1; g < q->g; g++) if (fin[g] < fin[best]) best = g;
-    fin[best] = fin[best] + (double)P->t[i * P->lp + l100];
+    fin[best] = fin[best] + t;
   }
   double T = 0.0;
   for (int g = 0; g < q->g; g++) if (fin[g] > T) T = fin[g];
   double E = 0.0;
-  for (int i = 0; i < q->n; i++)
-    E = E + (double)P->p[i * P->lp + l100] * (double)P->t[i * P->lp + l100];
+  if (q->model & OR_COUNT_IDLE) {
+    double D = 0.0;
+    for (int i = 0; i < q->n; i++)
+      D = D + ((double)P->p[i * P->lp + l100] - ps) * (double)P->t[i * P->lp + l100];
+    E = ((double)q->g * ps) * T + D;
+  } else {
+    for (int i = 0; i < q->n; i++) {
+      double t = (double)P->t[i * P->lp + l100], p = (double)P->p[i * P->lp + l100];
+      double e = p * t;
+      if (q->model & OR_POWER_CAP) {
+        double dyn = (p - ps) * t, tc = dyn / capd;
+        if (tc > t) e = ps * tc + dyn;
+      }
+      E = E + e;
+    }
+  }
   *tseq = T; *eseq = E;
 }
 
 /* ------------------------------------------------------------------ score */
-/* a[i]: group of workflow i; k groups; pl[i]: PROFILE level index of i.
- * returns 1 if feasible (T,E filled), 0 otherwise. */
-int oracle_score_config(const or_profile *P, int n, const int *a, int k,
+/* a[i]: group of workflow i; k groups; pl[i]: PROFILE level index of i;
+ * q: G and the model variant bits.  returns 1 if feasible (T,E filled), 0
+ * otherwise. */
+int oracle_score_config(const or_profile *P, const or_query *q, int n, const int *a, int k,
                         const int *pl, double *Tout, double *Eout) {
   const int lp = P->lp;
   for (int g = 0; g < k; g++) {
@@ -166,13 +213,15 @@ int oracle_score_config(const or_profile *P, int n, const int *a, int k,
     if (M > (long long)P->mem_cap) return 0;
   }
   const double ps = (double)P->ps;
-  double T = 0.0, E = 0.0;
+  const double capd = (double)q->power_cap - ps;
+  double T = 0.0, E = 0.0, Dall = 0.0;
   for (int g = 0; g < k; g++) {
     double U = 0.0, B = 0.0;
     for (int i = 0; i < n; i++) if (a[i] == g) {
       U = U + (double)P->u[i * lp + pl[i]];
       B = B + (double)P->bw[i * lp + pl[i]];
     }
+    if ((q->model & OR_NO_INTERFERENCE) && (U > 1.0 || B > 1.0)) return 0;
     double c = 1.0;
     if (U > c) c = U;
     if (B > c) c = B;
@@ -189,10 +238,16 @@ int oracle_score_config(const or_profile *P, int n, const int *a, int k,
       double dyn = ((double)P->p[i * lp + pl[i]] - ps) * (double)P->t[i * lp + pl[i]];
       D = D + dyn;
     }
+    if (q->model & OR_POWER_CAP) {
+      double tc = D / capd;
+      if (tc > Tg) Tg = tc;
+    }
     double Eg = ps * Tg + D;
     if (Tg > T) T = Tg;
     E = E + Eg;
+    Dall = Dall + D;
   }
+  if (q->model & OR_COUNT_IDLE) E = ((double)q->g * ps) * T + Dall;
   *Tout = T; *Eout = E;
   return 1;
 }
@@ -251,7 +306,7 @@ static void leaf(ctx_t *C, int k, uint64_t base) {
     }
     C->ncfg++;
     double T, E;
-    if (!oracle_score_config(C->P, q->n, C->a, k, pl, &T, &E)) continue;
+    if (!oracle_score_config(C->P, q, q->n, C->a, k, pl, &T, &E)) continue;
     C->nfeas++;
     for (int w = 0; w < q->nw; w++) {
       double F = objective(C->tseq, C->eseq, T, E, q->wa[w], q->wb[w]);

@@ -22,6 +22,8 @@ class Query:
     want_pareto: bool = True
     index_lo: int = 0
     index_hi: int | None = None   # None = |Omega|
+    model: int = 0                # scoring-model variant bits (R26-R28): 1 COUNT_IDLE,
+    power_cap: float = 0.0        # 2 NO_INTERFERENCE, 4 POWER_CAP (P_cap in W)
 
     def with_range(self, lo, hi):
         return dataclasses.replace(self, index_lo=lo, index_hi=hi)
