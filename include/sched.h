@@ -60,6 +60,21 @@ enum {
 
 enum { SCHED_PER_CLIENT = 0, SCHED_PER_GPU = 1 };
 
+/* Scoring-model variants (sched_query.model_flags; readings
+ * R26-R28 in DESIGN.md).  0 = the canonical model.
+ *  COUNT_IDLE       every one of the g GPUs draws the static power P_s for
+ *                   the whole makespan: E = g*P_s*T + sum_g D_g, and the
+ *                   sequential baseline E_seq = g*P_s*T_seq + sum_i dyn_i (R8 variant).
+ *  NO_INTERFERENCE  the PAPER.md L87 interference predicate as a hard rule
+ *                   (criterion 2, L90): a group whose combined SM or combined
+ *                   memory-BW utilisation exceeds 100 % is infeasible.
+ *  POWER_CAP        software power capping at power_cap_w (PAPER.md L162:
+ *                   300 W on A100X): a group is throttled until its average
+ *                   power is <= P_cap with its dynamic energy conserved,
+ *                   T_g' = max(T_g, D_g / (P_cap - P_s)); solo tasks of the
+ *                   sequential baseline likewise. */
+enum { SCHED_MODEL_COUNT_IDLE = 1, SCHED_MODEL_NO_INTERFERENCE = 2, SCHED_MODEL_POWER_CAP = 4 };
+
 #define SCHED_MAX_WORKFLOWS 32
 #define SCHED_MAX_GPUS 16
 #define SCHED_MAX_PROFILE_LEVELS 32
@@ -103,6 +118,8 @@ typedef struct {
   int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 12..40 (0 = default 22) */
   int32_t want_pareto;          /* nonzero: also compute the (T, E) Pareto set */
   uint32_t candidate_cap;       /* device Pareto-candidate buffer records; 0 = 1<<20 */
+  uint32_t model_flags;         /* SCHED_MODEL_* bits; 0 = canonical model */
+  float power_cap_w;            /* P_cap > P_s for SCHED_MODEL_POWER_CAP (else ignored) */
 } sched_query;
 
 /* One configuration and its scores.  score64/x64/y64/makespan_s/energy_j are

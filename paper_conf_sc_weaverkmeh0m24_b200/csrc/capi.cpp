@@ -44,6 +44,7 @@ int resolve(sched_handle *h, const sched_query *qin, Query *q, const Space **sp)
   int st = resolve_query_shape(qin, h->P.lp, q);
   if (st) return st;
   if (q->n > h->P.n) return SCHED_E_INVALID;
+  if ((q->model & SCHED_MODEL_POWER_CAP) && !(q->pcap > h->P.ps)) return SCHED_E_INVALID;  // R28
   st = get_space(h, *q, sp);
   if (st) return st;
   if (q->hi == UINT64_MAX || q->hi > (*sp)->total) q->hi = (*sp)->total;

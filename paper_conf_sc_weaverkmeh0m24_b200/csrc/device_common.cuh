@@ -80,10 +80,21 @@ __device__ __forceinline__ void stage_blob(unsigned char *sm, const DevParams &p
 //           exact T is read back from the candidate buffer slot.
 // Equal-T ties (configurations sharing a bottleneck group) are therefore
 // screened exactly.  All updates are monotone minima (race-free merges).
+//   pe[j] = min EXACT fp64 E (bits) over points in buckets < j: a configuration
+//           with exact (T, E), T in bucket j, is dominated if E >= pe[j]
+//           (exact ties in E, e.g. the constant-energy plateaus of the power
+//           cap model R28, are screened exactly).
 struct Stair {
   unsigned int *pm;
   unsigned long long *bp;
+  unsigned long long *pe;
 };
+
+// the CTA staircase in shared memory at `base` (kStairSmem bytes)
+__device__ __forceinline__ Stair stair_at(unsigned char *base) {
+  return Stair{(unsigned int *)(base + 16 * kBuckets), (unsigned long long *)base,
+               (unsigned long long *)(base + 8 * kBuckets)};
+}
 
 __device__ __forceinline__ int bucket_of(double T, uint32_t base) {
   const int b = (int)((unsigned long long)__double_as_longlong(T) >> kBucketShift) - (int)base;
@@ -94,6 +105,7 @@ __device__ __forceinline__ void stair_init(Stair s) {
   for (int i = threadIdx.x; i < kBuckets; i += blockDim.x) {
     s.pm[i] = 0x7f800000u;
     s.bp[i] = ~0ull;
+    s.pe[i] = ~0ull;
   }
 }
 
@@ -120,6 +132,21 @@ __device__ __forceinline__ void stair_merge(Stair s, const DevParams &p) {
     if (run < s.pm[j0 + k]) atomicMin(s.pm + j0 + k, run);
     run = min(run, __ldcg(p.stv + j0 + k));
   }
+  // exact-E prefix minima
+  unsigned long long te = ~0ull;
+  for (int k = 0; k < K; k++) te = min(te, __ldcg(p.ste + j0 + k));
+  unsigned long long pre_e = te;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long x = __shfl_up_sync(0xffffffffu, pre_e, o);
+    if (lane >= o) pre_e = min(pre_e, x);
+  }
+  unsigned long long run_e = __shfl_up_sync(0xffffffffu, pre_e, 1);
+  if (lane == 0) run_e = ~0ull;
+  for (int k = 0; k < K; k++) {
+    if (run_e < s.pe[j0 + k]) atomicMin(s.pe + j0 + k, run_e);
+    run_e = min(run_e, __ldcg(p.ste + j0 + k));
+  }
   __threadfence_block();
   __syncwarp();
 }
@@ -138,6 +165,22 @@ __device__ __forceinline__ bool stair_dominated(const Stair &s, const DevParams 
   return false;
 }
 
+// Exact domination of a configuration with exact canonical (T, E) by a
+// verified point: one in a strictly lower T bucket with E_p <= E, or the
+// bucket's recorded point.  Sound (only verified points), used after the
+// fp64 re-score, before a candidate is emitted.
+__device__ __forceinline__ bool stair_dominated_exact(const Stair &s, const DevParams &p, double T, double E) {
+  const int j = bucket_of(T, p.bucket_base);
+  if ((unsigned long long)__double_as_longlong(E) >= s.pe[j]) return true;
+  const unsigned long long pr = s.bp[j];
+  if ((unsigned int)pr != 0xffffffffu) {
+    const CandRec *c = (const CandRec *)p.cand + (unsigned int)pr;
+    const double ct = __ldcg(&c->t), ce = __ldcg(&c->e);
+    return ct <= T && ce <= E && (ct < T || ce < E);
+  }
+  return false;
+}
+
 // ---------------------------------------------------------- fp64 refine
 // Canonical score in fp64: explicit
 // round-to-nearest intrinsics, no contraction, same order as the oracle.
@@ -145,7 +188,7 @@ __device__ __forceinline__ bool stair_dominated(const Stair &s, const DevParams 
 __device__ __forceinline__ void refine64(const Tables &tb, const DevParams &p, const uint32_t *members,
                                          int k, const int *lam, double *Tout, double *Eout) {
   const double ps = p.ps;
-  double T = 0.0, E = 0.0;
+  double T = 0.0, E = 0.0, Dall = 0.0;
   for (int g = 0; g < k; g++) {
     const uint32_t m = members[g];
     double U = 0.0, B = 0.0;
@@ -173,12 +216,34 @@ __device__ __forceinline__ void refine64(const Tables &tb, const DevParams &p, c
       const int i = __ffs(mm) - 1, r = i * p.L + lam[i];
       D = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]));
     }
+    if (p.model & SCHED_MODEL_POWER_CAP) {  // R28
+      const double tc = __ddiv_rn(D, p.capd);
+      if (tc > Tg) Tg = tc;
+    }
     const double Eg = __dadd_rn(__dmul_rn(ps, Tg), D);
     if (Tg > T) T = Tg;
     E = __dadd_rn(E, Eg);
+    Dall = __dadd_rn(Dall, D);
   }
+  if (p.model & SCHED_MODEL_COUNT_IDLE) E = __dadd_rn(__dmul_rn(p.gps, T), Dall);  // R26
   *Tout = T;
   *Eout = E;
+}
+
+// R27 (NO_INTERFERENCE): every group's combined SM and BW utilisation, summed
+// in fp64 in ascending member order exactly as the oracle, is <= 1.
+__device__ __forceinline__ bool no_interference64(const Tables &tb, const DevParams &p, const uint32_t *members,
+                                                  int k, const int *lam) {
+  for (int g = 0; g < k; g++) {
+    double U = 0.0, B = 0.0;
+    for (uint32_t mm = members[g]; mm; mm &= mm - 1) {
+      const int i = __ffs(mm) - 1, r = i * p.L + lam[i];
+      U = __dadd_rn(U, (double)tb.u[r]);
+      B = __dadd_rn(B, (double)tb.bw[r]);
+    }
+    if (U > 1.0 || B > 1.0) return false;
+  }
+  return true;
 }
 
 __device__ __forceinline__ double objective64(const DevParams &p, double T, double E, int a, int b) {
@@ -248,6 +313,13 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
       improved = true;
     }
     atomicMin(s.bp + jb, pr);
+    const unsigned long long eb = (unsigned long long)__double_as_longlong(E);
+    if (eb < __ldcg(p.ste + jb)) {
+      atomicMin(p.ste + jb, eb);
+      improved = true;
+    }
+    const int hie = jb + 64 < kBuckets ? jb + 64 : kBuckets;
+    for (int i = jb + 1; i < hie; i++) atomicMin(s.pe + i, eb);
   } else {
     atomicExch(p.ctr + kCtrOverflow, 1ull);
   }
@@ -301,14 +373,26 @@ __device__ __forceinline__ void stair_sync(Stair s, const DevParams &p, u64 &pos
       if (need) atomicMin(s.pm + i, vb);
       if (__ballot_sync(0xffffffffu, need) != 0xffffffffu) break;
     }
+    if ((unsigned int)pr != 0xffffffffu) {  // exact E of the recorded point
+      unsigned long long eb = 0;
+      if (lane == 0) eb = (unsigned long long)__double_as_longlong(__ldcg(&((const CandRec *)p.cand + (unsigned int)pr)->e));
+      eb = __shfl_sync(0xffffffffu, eb, 0);
+      for (int i0 = (int)jb + 1; i0 < kBuckets; i0 += 32) {  // pe is non-increasing as well
+        const int i = i0 + lane;
+        const bool need = i < kBuckets && s.pe[i] > eb;
+        if (need) atomicMin(s.pe + i, eb);
+        if (__ballot_sync(0xffffffffu, need) != 0xffffffffu) break;
+      }
+    }
   }
   pos = ver;
   __syncwarp();
 }
 
 // fp32 tuple + exact canonical fp64 (T_g, E_g) of group `m` with every member
-// at level mu (canonical order of DESIGN.md section 2, as in refine64)
-__device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p, uint32_t m, int mu,
+// at level mu (canonical order of DESIGN.md section 2, as in refine64).
+// Returns false if the group is infeasible under NO_INTERFERENCE (R27).
+__device__ __forceinline__ bool group_eval(const Tables &tb, const DevParams &p, uint32_t m, int mu,
                                            float &t32, float &e32, double &t64, double &e64) {
   const int L = p.L;
   float U = 0.f, B = 0.f, D = 0.f;
@@ -321,6 +405,7 @@ __device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p,
     U64 = __dadd_rn(U64, (double)tb.u[r]);
     B64 = __dadd_rn(B64, (double)tb.bw[r]);
   }
+  if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (U64 > 1.0 || B64 > 1.0)) return false;
   const float cg = fmaxf(fmaxf(1.f, U), B);
   double c = 1.0;
   if (U64 > c) c = U64;
@@ -344,10 +429,16 @@ __device__ __forceinline__ void group_eval(const Tables &tb, const DevParams &p,
     const int r = (__ffs(mm) - 1) * L + mu;
     D64 = __dadd_rn(D64, __dmul_rn(__dsub_rn((double)tb.praw[r], p.ps), (double)tb.traw[r]));
   }
+  if (p.model & SCHED_MODEL_POWER_CAP) {  // R28: throttled to P_cap, dynamic energy conserved
+    Tg = fmaxf(Tg, D * p.kcap);
+    const double tc = __ddiv_rn(D64, p.capd);
+    if (tc > Tg64) Tg64 = tc;
+  }
   t32 = Tg;
   e32 = p.phat * Tg + D;
   t64 = Tg64;
   e64 = __dadd_rn(__dmul_rn(p.ps, Tg64), D64);
+  return true;
 }
 
 // ------------------------------------------------------------ DP walk (RGS state)

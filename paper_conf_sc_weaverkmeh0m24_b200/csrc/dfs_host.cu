@@ -24,6 +24,7 @@ static bool ws_match_d(const DevParams &dp, int *perm) {
 
 bool dfs_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.L != 1 || dp.g > kDfsMaxG || dp.c > kDfsMaxC || dp.n < 4 || !dp.gtab_ok) return false;
+  if (dp.model & SCHED_MODEL_COUNT_IDLE) return false;  // E = sum_g E_g only
   int perm[kMaxW];
   const void *fn = nullptr;
 #define TRY(WS)                                                    \
@@ -39,7 +40,7 @@ bool dfs_eligible(DevParams &dp, TileLaunch *tl) {
 #undef TRY
   if (!fn) return false;
   tl->fn = fn;
-  tl->smem = ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(PairWarp) * (kDfsThreads / 32) +
+  tl->smem = ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(PairWarp) * (kDfsThreads / 32) +
              sizeof(BestRec) * (kDfsThreads / 32) * kMaxW + sizeof(float) * kDfsThreads * kMaxW;
   return true;
 }

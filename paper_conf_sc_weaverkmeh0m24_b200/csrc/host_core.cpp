@@ -97,6 +97,11 @@ int resolve_query_shape(const sched_query *q, int n_profile_levels, Query *Q) {
   Q->cand_cap = q->candidate_cap == 0 ? (1u << 20) : q->candidate_cap;
   Q->lo = q->index_lo;
   Q->hi = q->index_hi;
+  if (q->model_flags & ~(uint32_t)(SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE | SCHED_MODEL_POWER_CAP))
+    return SCHED_E_INVALID;
+  Q->model = q->model_flags;
+  Q->pcap = q->power_cap_w;
+  if ((Q->model & SCHED_MODEL_POWER_CAP) && !(std::isfinite(Q->pcap) && Q->pcap > 0.f)) return SCHED_E_INVALID;
   return SCHED_OK;
 }
 
@@ -105,6 +110,7 @@ int resolve_query(const Profile *P, const sched_query *q, Query *Q, uint64_t *to
   int st = resolve_query_shape(q, P->lp, Q);
   if (st) return st;
   if (Q->n > P->n) return SCHED_E_INVALID;
+  if ((Q->model & SCHED_MODEL_POWER_CAP) && !(Q->pcap > P->ps)) return SCHED_E_INVALID;
   Space sp;
   st = build_space(*Q, &sp);
   if (st) return st;
@@ -306,21 +312,44 @@ int host_rank(const Space &sp, const int8_t *a, const int8_t *digits, uint64_t *
 // Sequential baseline ("jobs are scheduled individually on GPUs
 // in queue order with no parallel overlap"; R6, R16): list schedule at 100%.
 void host_constants(const Profile &P, const Query &q, double *tseq, double *eseq) {
+  const double ps = (double)P.ps, capd = (double)q.pcap - ps;
+  const bool cap = q.model & SCHED_MODEL_POWER_CAP;
   double fin[kMaxG];
   for (int g = 0; g < q.g; g++) fin[g] = 0.0;
   for (int i = 0; i < q.n; i++) {
+    const size_t k = (size_t)i * P.lp + P.l100;
+    double t = (double)P.t[k];
+    if (cap) {  // R28: a solo task above P_cap runs dyn / (P_cap - P_s)
+      const double tc = (((double)P.p[k] - ps) * t) / capd;
+      if (tc > t) t = tc;
+    }
     int best = 0;
     for (int g = 1; g < q.g; g++)
       if (fin[g] < fin[best]) best = g;
-    fin[best] = fin[best] + (double)P.t[(size_t)i * P.lp + P.l100];
+    fin[best] = fin[best] + t;
   }
   double T = 0.0;
   for (int g = 0; g < q.g; g++)
     if (fin[g] > T) T = fin[g];
   double E = 0.0;
-  for (int i = 0; i < q.n; i++) {
-    const size_t k = (size_t)i * P.lp + P.l100;
-    E = E + (double)P.p[k] * (double)P.t[k];
+  if (q.model & SCHED_MODEL_COUNT_IDLE) {  // R26: E_seq = g P_s T_seq + sum dyn
+    double D = 0.0;
+    for (int i = 0; i < q.n; i++) {
+      const size_t k = (size_t)i * P.lp + P.l100;
+      D = D + ((double)P.p[k] - ps) * (double)P.t[k];
+    }
+    E = ((double)q.g * ps) * T + D;
+  } else {
+    for (int i = 0; i < q.n; i++) {
+      const size_t k = (size_t)i * P.lp + P.l100;
+      const double t = (double)P.t[k], p = (double)P.p[k];
+      double e = p * t;
+      if (cap) {
+        const double dyn = (p - ps) * t, tc = dyn / capd;
+        if (tc > t) e = ps * tc + dyn;
+      }
+      E = E + e;
+    }
   }
   *tseq = T;
   *eseq = E;
@@ -340,7 +369,7 @@ int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const i
     if (M > (long long)P.mem_cap) return 0;
   }
   const double ps = (double)P.ps;
-  double T = 0.0, E = 0.0;
+  double T = 0.0, E = 0.0, Dall = 0.0;
   for (int g = 0; g < k; g++) {
     double U = 0.0, B = 0.0;
     for (int i = 0; i < n; i++)
@@ -348,6 +377,7 @@ int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const i
         U = U + (double)P.u[(size_t)i * lp + pl[i]];
         B = B + (double)P.bw[(size_t)i * lp + pl[i]];
       }
+    if ((q.model & SCHED_MODEL_NO_INTERFERENCE) && (U > 1.0 || B > 1.0)) return 0;  // R27
     double c = 1.0;
     if (U > c) c = U;
     if (B > c) c = B;
@@ -367,10 +397,16 @@ int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const i
         const size_t r = (size_t)i * lp + pl[i];
         D = D + ((double)P.p[r] - ps) * (double)P.t[r];
       }
+    if (q.model & SCHED_MODEL_POWER_CAP) {  // R28
+      const double tc = D / ((double)q.pcap - ps);
+      if (tc > Tg) Tg = tc;
+    }
     const double Eg = ps * Tg + D;
     if (Tg > T) T = Tg;
     E = E + Eg;
+    Dall = Dall + D;
   }
+  if (q.model & SCHED_MODEL_COUNT_IDLE) E = ((double)q.g * ps) * T + Dall;  // R26
   *Tout = T;
   *Eout = E;
   return 1;
@@ -410,6 +446,11 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->tseq = tseq;
   dp->eseq = eseq;
   dp->phat = (float)((double)P.ps * tseq / eseq);
+  dp->model = q.model;
+  dp->capd = (double)q.pcap - (double)P.ps;
+  dp->kcap = (q.model & SCHED_MODEL_POWER_CAP) ? (float)(eseq / (dp->capd * tseq)) : 0.f;
+  dp->gps = (double)q.g * (double)P.ps;
+  dp->kidle = (float)(dp->gps * tseq / eseq);
   dp->mem_cap = P.mem_cap;
   dp->want_pareto = q.want_pareto;
   for (int w = 0; w < q.nw; w++) {

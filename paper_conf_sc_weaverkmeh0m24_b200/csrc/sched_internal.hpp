@@ -20,6 +20,7 @@ constexpr int kBuckets = 2048;                  // Pareto staircase buckets (per
 constexpr int kBucketShift = 45;                // of the fp64 bits of T: 128 buckets per binade
 constexpr uint16_t kNoState = 0xFFFF;
 constexpr int kUnitLog2 = 11;
+constexpr int kStairSmem = 20 * kBuckets;       // per-CTA staircase: bp, pe (u64) + pm (u32) per bucket
 constexpr int kLog = 4096;                      // staircase insertion log (ring buffer entries)                   // generic kernel: 2048 configs per warp unit
 
 // Validated host copy of sched_profile.
@@ -42,6 +43,8 @@ struct Query {
   int rank, count, chunk_log2;
   int want_pareto;
   uint32_t cand_cap;
+  uint32_t model;           // SCHED_MODEL_* bits
+  float pcap;               // P_cap (W) for SCHED_MODEL_POWER_CAP
 };
 
 // DP count table (host + device): state = (elements placed, open groups,
@@ -71,6 +74,11 @@ struct DevParams {
   float tlb_scale_f;        // the same, as a float rounded down
   float phat;               // P_s * T_seq / E_seq
   double ps, tseq, eseq;
+  uint32_t model;           // SCHED_MODEL_* bits (R26-R28)
+  double capd;              // P_cap - P_s (exact) for POWER_CAP
+  float kcap;               // E_seq / ((P_cap - P_s) T_seq): normalised capped time = D-hat * kcap
+  float kidle;              // g P_s T_seq / E_seq: COUNT_IDLE energy term per normalised T
+  double gps;               // g * P_s (exact) for COUNT_IDLE
   int mem_cap, want_pareto, root, nstates;
   uint32_t bucket_base;     // (bits64(T_lower) >> kBucketShift)
   // work split
@@ -90,6 +98,7 @@ struct DevParams {
   unsigned int *thr;           // [kMaxW] global fp32 proxy threshold bits (min)
   unsigned int *stv;           // [kBuckets] min val of verified points per bucket
   unsigned long long *stp;     // [kBuckets] min (val << 32 | candidate slot) per bucket
+  unsigned long long *ste;     // [kBuckets] min exact E (fp64 bits) of the verified points per bucket
   unsigned char *stlog;        // [kLog] LogEnt: insertion log (seq = ctr[kCtrStairVer])
   unsigned char *slots;        // [grid][W] BestRec
   unsigned char *cand;         // [cand_cap] CandRec

@@ -39,6 +39,7 @@ __device__ __forceinline__ void score32(const Tables &tb, const DevParams &p, co
                                         const int *lam, float &T, float &E) {
   T = 0.f;
   E = 0.f;
+  float Dall = 0.f;
   for (int g = 0; g < c.k; g++) {
     const uint32_t m = c.mask[g];
     float U = 0.f, B = 0.f, D = 0.f;
@@ -56,9 +57,12 @@ __device__ __forceinline__ void score32(const Tables &tb, const DevParams &p, co
       for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) s += tb.d[ri * p.ds + (__ffs(m2) - 1) * p.L + lam[__ffs(m2) - 1]];
       Tg = fmaxf(Tg, tb.th[ri] * s * cg);
     }
+    if (p.model & SCHED_MODEL_POWER_CAP) Tg = fmaxf(Tg, D * p.kcap);  // R28
     T = fmaxf(T, Tg);
     E += p.phat * Tg + D;
+    Dall += D;
   }
+  if (p.model & SCHED_MODEL_COUNT_IDLE) E = p.kidle * T + Dall;  // R26
 }
 
 __device__ __forceinline__ float proxy(float T, float E, int a, int b) {
@@ -78,8 +82,8 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
   const Tables tb = tables_at(sm, p);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
-  Stair stair{(unsigned int *)(after + 8 * kBuckets), (unsigned long long *)after};
-  BestRec *red = (BestRec *)(after + 12 * kBuckets);
+  Stair stair = stair_at(after);
+  BestRec *red = (BestRec *)(after + kStairSmem);
   stair_init(stair);
   __syncthreads();
   u64 stair_ver = 0;
@@ -124,7 +128,12 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
     if (idx < lend && dev_unrank(tb, p, idx, c)) {
       for (;;) {
         ncfg++;
-        if (c.feasible) {
+        bool feas = c.feasible;
+        if (feas && (p.model & SCHED_MODEL_NO_INTERFERENCE)) {  // level-dependent (R27)
+          decode_levels(p, c, lam);
+          feas = no_interference64(tb, p, c.mask, c.k, lam);
+        }
+        if (feas) {
           nfeas++;
           decode_levels(p, c, lam);
           float T, E;
@@ -165,7 +174,8 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
                 }
               }
             }
-            if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))))
+            if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))) &&
+                !stair_dominated_exact(stair, p, T64, E64))
               emit_candidate(p, stair, idx, T64, E64, T, E);
           }
         }
@@ -231,7 +241,7 @@ __global__ void __launch_bounds__(256) k_groups(const DevParams p, GroupRec *gta
        id += (unsigned long long)gridDim.x * blockDim.x) {
     const uint32_t m = (uint32_t)(id / p.L);
     const int mu = (int)(id % p.L);
-    GroupRec r;
+    GroupRec r, x;
     r.t32 = __int_as_float(0x7f800000);
     r.e32 = 0.f;
     r.t64 = __longlong_as_double(0x7ff0000000000000ll);
@@ -239,7 +249,7 @@ __global__ void __launch_bounds__(256) k_groups(const DevParams p, GroupRec *gta
     if (m != 0 && __popc(m) <= p.c) {
       long long M = 0;
       for (uint32_t mm = m; mm; mm &= mm - 1) M += tb.mem[__ffs(mm) - 1];
-      if (M <= (long long)p.mem_cap) group_eval(tb, p, m, mu, r.t32, r.e32, r.t64, r.e64);
+      if (M <= (long long)p.mem_cap && group_eval(tb, p, m, mu, x.t32, x.e32, x.t64, x.e64)) r = x;
     }
     gtab[id] = r;
   }
@@ -262,6 +272,7 @@ __global__ void k_init(const DevParams p, int keep) {
   for (int i = t; i < kBuckets; i += blockDim.x) {
     p.stv[i] = 0x7f800000u;
     p.stp[i] = ~0ull;
+    p.ste[i] = ~0ull;
   }
 }
 
@@ -329,15 +340,16 @@ __global__ void k_best_final(const DevParams p, int nslots) {
 // verified point of the final global staircase; compact survivors.
 __global__ void k_pareto_prefilter(const DevParams p, int ncand, unsigned int *surv) {
   __shared__ unsigned int s_pm[kBuckets];
-  __shared__ unsigned long long s_bp[kBuckets];
-  Stair stair{s_pm, s_bp};
+  __shared__ unsigned long long s_bp[kBuckets], s_pe[kBuckets];
+  Stair stair{s_pm, s_bp, s_pe};
   stair_init(stair);
   __syncthreads();
   if (threadIdx.x < 32) stair_merge(stair, p);
   __syncthreads();
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
     const CandRec c = ((const CandRec *)p.cand)[i];
-    const bool dom = stair_dominated(stair, p, c.t, __double2float_rd(__ddiv_rd(c.e, p.eseq)));
+    const bool dom = stair_dominated(stair, p, c.t, __double2float_rd(__ddiv_rd(c.e, p.eseq))) ||
+                     stair_dominated_exact(stair, p, c.t, c.e);
     if (!dom) {
       const unsigned int k = (unsigned int)atomicAdd(p.ctr + kCtrSurv, 1ull);
       surv[k] = (unsigned int)i;
@@ -409,7 +421,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, stlog, blob, slots, cand, surv, keep, out, gtab, total;
+  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, keep, out, gtab, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -425,6 +437,7 @@ WsLayout layout(const DevParams &dp) {
   L.thr = take(4 * kMaxW);
   L.stv = take(4 * kBuckets);
   L.stp = take(8 * kBuckets);
+  L.ste = take(8 * kBuckets);
   L.stlog = take(sizeof(LogEnt) * kLog);
   L.blob = take(dp.blob_bytes);
   L.slots = take(sizeof(BestRec) * kMaxW * (size_t)kMaxGrid);
@@ -471,6 +484,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.thr = (unsigned int *)(ws + L.thr);
   dp.stv = (unsigned int *)(ws + L.stv);
   dp.stp = (unsigned long long *)(ws + L.stp);
+  dp.ste = (unsigned long long *)(ws + L.ste);
   dp.stlog = ws + L.stlog;
   dp.slots = ws + L.slots;
   dp.cand = ws + L.cand;
@@ -540,7 +554,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       path = 2;
       CK(launch_dfs(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
     } else {
-      const size_t smem = ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(BestRec) * kWarps * kMaxW;
+      const size_t smem = ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(BestRec) * kWarps * kMaxW;
       CK(cudaFuncSetAttribute(k_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       int occ = 0;
       CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_generic, kThreads, smem));

@@ -194,7 +194,8 @@ __device__ __noinline__ int pair_slow(const Tables &tb, const DevParams &p, cons
         }
       }
     }
-    if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))))
+    if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))) &&
+        !stair_dominated_exact(stair, p, T64, E64))
       emit_candidate(p, stair, idx, T64, E64, T, E);
   }
   return nref;
@@ -207,8 +208,8 @@ __global__ void __launch_bounds__(kDfsThreads, 2) k_dfs(const DevParams p) {
   const Tables tb = tables_at(sm, p);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
-  Stair stair{(unsigned int *)(after + 8 * kBuckets), (unsigned long long *)after};
-  PairWarp *pws = (PairWarp *)(after + 12 * kBuckets);
+  Stair stair = stair_at(after);
+  PairWarp *pws = (PairWarp *)(after + kStairSmem);
   PairWarp &w = pws[warp];
   BestRec *red = (BestRec *)(pws + kDfsThreads / 32);
   float *thr_sm = (float *)(red + (kDfsThreads / 32) * kMaxW) + threadIdx.x * kMaxW;

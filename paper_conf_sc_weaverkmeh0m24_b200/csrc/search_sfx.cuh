@@ -140,7 +140,8 @@ static __device__ __noinline__ void sfx_check(const DevParams &p, const Stair &s
       }
     }
   }
-  if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))))
+  if (par && !stair_dominated(stair, p, T64, __double2float_rd(__ddiv_rd(E64, p.eseq))) &&
+      !stair_dominated_exact(stair, p, T64, E64))
     emit_candidate(p, stair, idx, T64, E64, T, E);
 }
 
@@ -470,8 +471,8 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
   constexpr int RS = SfxWarp<M>::RS;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
-  Stair stair{(unsigned int *)(after + 8 * kBuckets), (unsigned long long *)after};
-  SfxWarp<M> *wps = (SfxWarp<M> *)(after + 12 * kBuckets);
+  Stair stair = stair_at(after);
+  SfxWarp<M> *wps = (SfxWarp<M> *)(after + kStairSmem);
   SfxWarp<M> &w = wps[warp];
   BestRec *red = (BestRec *)(wps + kSfxWarps);
   stair_init(stair);

@@ -154,7 +154,8 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
       }
     }
   }
-  if (par && !stair_dominated(stair, p, T64r, __double2float_rd(__ddiv_rd(E64, p.eseq))))
+  if (par && !stair_dominated(stair, p, T64r, __double2float_rd(__ddiv_rd(E64, p.eseq))) &&
+      !stair_dominated_exact(stair, p, T64r, E64))
     emit_candidate(p, stair, idx, T64r, E64, T, E);
   return 1;
 }
@@ -367,8 +368,8 @@ __global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
   const Tables tb = tables_at(sm, p);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
-  Stair stair{(unsigned int *)(after + 8 * kBuckets), (unsigned long long *)after};
-  WarpPart *wps = (WarpPart *)(after + 12 * kBuckets);
+  Stair stair = stair_at(after);
+  WarpPart *wps = (WarpPart *)(after + kStairSmem);
   WarpPart &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kTileWarps);
   float *thr_sm = (float *)(red + kTileWarps * kMaxW) + threadIdx.x * kMaxW;

@@ -6,11 +6,12 @@ namespace sched {
 
 static size_t sfx_smem(const DevParams &dp, int M) {
   const size_t warp = M == 6 ? sizeof(SfxWarp<6>) : sizeof(SfxWarp<4>);
-  return ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + warp * kSfxWarps + sizeof(BestRec) * kSfxWarps * kMaxW;
+  return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + warp * kSfxWarps + sizeof(BestRec) * kSfxWarps * kMaxW;
 }
 
 bool sfx_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.L != 1 || dp.g > kSfxMaxG || (dp.capped && dp.c > 15) || !dp.gtab_ok) return false;
+  if (dp.model & SCHED_MODEL_COUNT_IDLE) return false;  // E = sum_g E_g only
   int M;
   if (dp.n >= 8) M = 6;
   else if (dp.n >= 6) M = 4;

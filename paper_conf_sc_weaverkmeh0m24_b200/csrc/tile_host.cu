@@ -39,12 +39,15 @@ static const void *tile_pick_ws(DevParams *dp) {
 }
 
 size_t tile_smem_bytes(const DevParams &dp) {
-  return ((dp.blob_bytes + 15) & ~15u) + 12 * kBuckets + sizeof(WarpPart) * kTileWarps +
+  return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(WarpPart) * kTileWarps +
          sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * kMaxW;
 }
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4 || !dp.gtab_ok) return false;
+  // E = sum_g E_g with level-independent feasibility: COUNT_IDLE (global
+  // energy term) and NO_INTERFERENCE (level-dependent feasibility) take the generic kernel
+  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE)) return false;
   const void *fn = tile_pick_ws<4>(&dp);
   if (!fn) return false;
   tl->fn = fn;

@@ -25,6 +25,9 @@ SCHED_E_WORKSPACE = -6
 SCHED_E_NODEVICE = -7
 PER_CLIENT = 0
 PER_GPU = 1
+SCHED_MODEL_COUNT_IDLE = 1        # scoring-model variants (include/sched.h, R26-R28)
+SCHED_MODEL_NO_INTERFERENCE = 2
+SCHED_MODEL_POWER_CAP = 4
 UINT64_MAX = (1 << 64) - 1
 
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
@@ -52,7 +55,8 @@ class _Query(C.Structure):
                 ("level_mask", C.c_uint32), ("level_scope", C.c_int32), ("n_weights", C.c_int32),
                 ("weights", C.POINTER(C.c_int32)), ("index_lo", C.c_uint64), ("index_hi", C.c_uint64),
                 ("shard_rank", C.c_int32), ("shard_count", C.c_int32), ("chunk_log2", C.c_int32),
-                ("want_pareto", C.c_int32), ("candidate_cap", C.c_uint32)]
+                ("want_pareto", C.c_int32), ("candidate_cap", C.c_uint32),
+                ("model_flags", C.c_uint32), ("power_cap_w", C.c_float)]
 
 
 class Pick(C.Structure):
@@ -164,7 +168,8 @@ class Scheduler:
         hi = UINT64_MAX if q.index_hi is None else int(q.index_hi)
         cq = _Query(q.n, q.g, q.c, mask, q.scope, len(q.weights), w.ctypes.data_as(C.POINTER(C.c_int32)),
                     int(q.index_lo), hi, int(shard[0]), int(shard[1]), int(chunk_log2),
-                    int(bool(q.want_pareto)), int(candidate_cap))
+                    int(bool(q.want_pareto)), int(candidate_cap), int(getattr(q, "model", 0)),
+                    float(getattr(q, "power_cap", 0.0)))
         cq._keep = w
         return cq
 
@@ -228,7 +233,7 @@ class Scheduler:
 
 def _shape_query(q):
     mask = (1 << len(q.levels)) - 1   # shape-only calls: only L = popcount matters
-    cq = _Query(q.n, q.g, q.c, mask, q.scope, 0, None, 0, UINT64_MAX, 0, 1, 22, 0, 0)
+    cq = _Query(q.n, q.g, q.c, mask, q.scope, 0, None, 0, UINT64_MAX, 0, 1, 22, 0, 0, 0, 0.0)
     return cq
 
 

@@ -89,6 +89,42 @@ def test_host_score_bitwise_oracle(name):
                 assert p.score64 == oracle.objective(ts, es, T, E, a, b)
 
 
+@pytest.mark.parametrize("model", [1, 2, 4, 7])
+@pytest.mark.parametrize("name", ["c2", "c4", "c5"])
+def test_host_score_variants_bitwise_oracle(name, model):
+    """Library fp64 host score (sched_score) under the scoring-model variants
+    (R26-R28) == the oracle's, bitwise, including the variant baselines."""
+    import dataclasses
+    prof, q = config(name)
+    q = dataclasses.replace(q, model=model, power_cap=180.0)
+    sch = S.Scheduler(prof)
+    tot = S.count(q)
+    rnd = random.Random(7)
+    ts, es = oracle.constants(prof, q)
+    nv = 0
+    for idx in [0, tot - 1] + [rnd.randrange(tot) for _ in range(40)]:
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, idx))
+        for w, (a, b) in enumerate(q.weights):
+            p = sch.score(q, idx, w)
+            assert p.valid == ok
+            if ok:
+                nv += 1
+                assert p.makespan_s == T and p.energy_j == E
+                assert p.score64 == oracle.objective(ts, es, T, E, a, b)
+    assert nv > 0 or model & 2   # c5 groups of 3 mostly exceed 100 % SM
+
+
+def test_variant_queries_validated():
+    """POWER_CAP needs P_cap > P_s; unknown model bits are rejected."""
+    import dataclasses
+    prof, q = config("c1")
+    sch = S.Scheduler(prof)
+    for bad in (dict(model=4, power_cap=50.0), dict(model=4, power_cap=0.0), dict(model=8)):
+        with pytest.raises(S.SchedError) as e:
+            sch.score(dataclasses.replace(q, **bad), 0, 0)
+        assert e.value.status == S.sched.SCHED_E_INVALID
+
+
 def test_invalid_profiles_rejected():
     prof = make_profile(4, levels=(50, 100), seed=1)
     bad = make_profile(4, levels=(50, 100), seed=1)
