@@ -96,8 +96,8 @@ __device__ __forceinline__ Stair stair_at(unsigned char *base) {
                (unsigned long long *)(base + 8 * kBuckets)};
 }
 
-__device__ __forceinline__ int bucket_of(double T, uint32_t base) {
-  const int b = (int)((unsigned long long)__double_as_longlong(T) >> kBucketShift) - (int)base;
+__device__ __forceinline__ int bucket_of(double T, const DevParams &p) {
+  const int b = (int)((unsigned long long)__double_as_longlong(T) >> p.bucket_shift) - (int)p.bucket_base;
   return b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
 }
 
@@ -154,7 +154,7 @@ __device__ __forceinline__ void stair_merge(Stair s, const DevParams &p) {
 // T: exact canonical fp64 makespan (or a lower bound of it that is itself an
 // exact canonical makespan); eh: fp32 normalised energy (or a lower bound).
 __device__ __forceinline__ bool stair_dominated(const Stair &s, const DevParams &p, double T, float eh) {
-  const int j = bucket_of(T, p.bucket_base);
+  const int j = bucket_of(T, p);
   const unsigned int eb = __float_as_uint(eh);
   if (eb > s.pm[j]) return true;
   const unsigned long long pr = s.bp[j];
@@ -170,7 +170,7 @@ __device__ __forceinline__ bool stair_dominated(const Stair &s, const DevParams 
 // bucket's recorded point.  Sound (only verified points), used after the
 // fp64 re-score, before a candidate is emitted.
 __device__ __forceinline__ bool stair_dominated_exact(const Stair &s, const DevParams &p, double T, double E) {
-  const int j = bucket_of(T, p.bucket_base);
+  const int j = bucket_of(T, p);
   if ((unsigned long long)__double_as_longlong(E) >= s.pe[j]) return true;
   const unsigned long long pr = s.bp[j];
   if ((unsigned int)pr != 0xffffffffu) {
@@ -292,7 +292,7 @@ __device__ __forceinline__ void emit_candidate(const DevParams &p, Stair s, u64 
   const double g1 = 1.0 + (double)p.gamma;
   const float val = __double2float_ru(__dmul_ru(__ddiv_ru(E, p.eseq), g1));
   const unsigned int vb = __float_as_uint(val);
-  const int jb = bucket_of(T, p.bucket_base);
+  const int jb = bucket_of(T, p);
   bool improved = false;
   if (vb < __ldcg(p.stv + jb)) {
     atomicMin(p.stv + jb, vb);

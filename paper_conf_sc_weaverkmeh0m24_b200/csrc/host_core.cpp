@@ -530,6 +530,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
     const double tl = (double)tlow * 0.5 * tseq;
     uint64_t b;
     std::memcpy(&b, &tl, 8);
+    dp->bucket_shift = kBucketShift;
     dp->bucket_base = (uint32_t)(b >> kBucketShift);
   }
   std::memcpy(B + dp->off_W, sp.W.data(), 8 * sp.W.size());

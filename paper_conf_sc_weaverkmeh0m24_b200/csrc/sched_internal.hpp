@@ -17,7 +17,8 @@ constexpr int kMaxG = SCHED_MAX_GPUS;           // 16
 constexpr int kMaxL = SCHED_MAX_SEARCH_LEVELS;  // 8
 constexpr int kMaxW = SCHED_MAX_WEIGHTS;        // 8
 constexpr int kBuckets = 2048;                  // Pareto staircase buckets (per CTA)
-constexpr int kBucketShift = 45;                // of the fp64 bits of T: 128 buckets per binade
+constexpr int kBucketShift = 45;                // of the fp64 bits of T: 128 buckets per binade (default)
+constexpr int kBucketShiftMin = 33;             // finest re-bucketing: 2^19 buckets per binade (>= 29: fp32 screen)
 constexpr uint16_t kNoState = 0xFFFF;
 constexpr int kUnitLog2 = 11;
 constexpr int kStairSmem = 20 * kBuckets;       // per-CTA staircase: bp, pe (u64) + pm (u32) per bucket
@@ -80,7 +81,8 @@ struct DevParams {
   float kidle;              // g P_s T_seq / E_seq: COUNT_IDLE energy term per normalised T
   double gps;               // g * P_s (exact) for COUNT_IDLE
   int mem_cap, want_pareto, root, nstates;
-  uint32_t bucket_base;     // (bits64(T_lower) >> kBucketShift)
+  uint32_t bucket_base;     // (bits64(T_lower) >> bucket_shift)
+  int bucket_shift;         // kBucketShift, or finer after the seed pass (re-bucketing, search.cu)
   // work split
   uint64_t lo, hi;          // window
   uint64_t first_chunk;     // first owned chunk id

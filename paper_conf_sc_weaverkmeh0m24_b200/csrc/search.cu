@@ -15,6 +15,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <cstring>
 
@@ -258,21 +259,71 @@ __global__ void __launch_bounds__(256) k_groups(const DevParams p, GroupRec *gta
 // ------------------------------------------------------------ init / finalize
 // keep = 0: fresh search; 1: seeded re-run after overflow (keep staircase +
 // thresholds, drop candidates); 2: after the seed pass (keep staircase,
-// thresholds and the seed pass's in-range candidates).
+// thresholds and the seed pass's in-range candidates); 3: after the seed pass
+// with a new staircase bucketing (keep thresholds and candidates, reset the
+// staircase, which k_rebucket then rebuilds from the candidates).
 __global__ void k_init(const DevParams p, int keep) {
   const int t = threadIdx.x;
   const bool kept = keep && (t == kCtrStairVer || t == kCtrPass ||
-                             (keep == 2 && (t == kCtrCand || t == kCtrOverflow)));
+                             (keep >= 2 && (t == kCtrCand || t == kCtrOverflow)));
   if (t < kCtrN && !kept) p.ctr[t] = 0ull;
   if (keep != 2)  // a fresh log (re-run: its slot ids are rewritten by k_reseed)
     for (int i = t; i < kLog; i += blockDim.x) ((LogEnt *)p.stlog)[i].tag = 0u;
-  if (keep == 1 && t == kCtrStairVer) p.ctr[t] = (unsigned long long)kLog + 1;  // forces a full merge
-  if (keep) return;
-  if (t < kMaxW) p.thr[t] = 0x7f800000u;
+  if ((keep == 1 || keep == 3) && t == kCtrStairVer) p.ctr[t] = (unsigned long long)kLog + 1;  // full merge
+  if (keep == 1 || keep == 2) return;
+  if (t < kMaxW && keep == 0) p.thr[t] = 0x7f800000u;
   for (int i = t; i < kBuckets; i += blockDim.x) {
     p.stv[i] = 0x7f800000u;
     p.stp[i] = ~0ull;
     p.ste[i] = ~0ull;
+  }
+}
+
+// Span of the verified points after the seed pass: out[0] = min T, out[1] =
+// the T of the lowest-energy point (the front's two ends).  One block.
+__global__ void __launch_bounds__(1024) k_stair_span(const DevParams p, int ncand, double *out) {
+  __shared__ double s_t[1024], s_e[1024], s_te[1024];
+  double tlo = __longlong_as_double(0x7ff0000000000000ll), emin = tlo, temin = tlo;
+  for (int i = threadIdx.x; i < ncand; i += blockDim.x) {
+    const CandRec c = ((const CandRec *)p.cand)[i];
+    tlo = fmin(tlo, c.t);
+    if (c.e < emin || (c.e == emin && c.t < temin)) {
+      emin = c.e;
+      temin = c.t;
+    }
+  }
+  s_t[threadIdx.x] = tlo;
+  s_e[threadIdx.x] = emin;
+  s_te[threadIdx.x] = temin;
+  __syncthreads();
+  for (int o = 512; o; o >>= 1) {
+    if (threadIdx.x < o) {
+      const int q = threadIdx.x + o;
+      s_t[threadIdx.x] = fmin(s_t[threadIdx.x], s_t[q]);
+      if (s_e[q] < s_e[threadIdx.x] || (s_e[q] == s_e[threadIdx.x] && s_te[q] < s_te[threadIdx.x])) {
+        s_e[threadIdx.x] = s_e[q];
+        s_te[threadIdx.x] = s_te[q];
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    out[0] = s_t[0];
+    out[1] = s_te[0];
+  }
+}
+
+// Re-insert the seed pass's candidate records into the staircase under the
+// new bucketing (same values as emit_candidate).
+__global__ void k_rebucket(const DevParams p, int ncand) {
+  const double g1 = 1.0 + (double)p.gamma;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < ncand; i += gridDim.x * blockDim.x) {
+    const CandRec c = ((const CandRec *)p.cand)[i];
+    const unsigned int vb = __float_as_uint(__double2float_ru(__dmul_ru(__ddiv_ru(c.e, p.eseq), g1)));
+    const int jb = bucket_of(c.t, p);
+    atomicMin(p.stv + jb, vb);
+    atomicMin(p.stp + jb, ((unsigned long long)vb << 32) | (unsigned int)i);
+    atomicMin(p.ste + jb, (unsigned long long)__double_as_longlong(c.e));
   }
 }
 
@@ -523,7 +574,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     search_ms += gms;
     launches++;
   }
-  const DevParams dp_full = dp;
+  DevParams dp_full = dp;
   const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
                     (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 26);  // >= 2^38 configs
   for (int pass = seed ? 0 : 1; pass < 3; pass++) {
@@ -535,9 +586,42 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       dp.unit_stride = u12 / dp.n_units;
     }
     passes++;
-    k_init<<<1, 256, 0, st>>>(dp, pass == 0 ? 0 : (pass == 1 ? (seed ? 2 : 0) : 1));
+    int keep = pass == 0 ? 0 : (pass == 1 ? (seed ? 2 : 0) : 1);
+    const int ncand0 = pass == 1 && seed && dp.want_pareto ? (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap) : 0;
+    if (ncand0 > 0) {
+      // Re-bucket the staircase to the span of the seed pass's front: about
+      // 1024 buckets between its lowest T and the T of its lowest-E point,
+      // so that front points closer than the default 2^-7 relative bucket
+      // width are screened exactly (dense local fronts of index windows).
+      double span[2];
+      k_stair_span<<<1, 1024, 0, st>>>(dp, ncand0, (double *)dp.out);
+      CK(cudaGetLastError());
+      CK(cudaMemcpyAsync(span, dp.out, sizeof span, cudaMemcpyDeviceToHost, st));
+      CK(cudaStreamSynchronize(st));
+      launches++;
+      d2h += sizeof span;
+      if (span[0] > 0.0 && span[1] >= span[0] && std::isfinite(span[1])) {
+        const double binades = std::log2(span[1] / span[0]);
+        int sh = (int)std::ceil(52.0 - std::log2(1024.0 / std::max(binades, 1e-9)));
+        sh = std::max(kBucketShiftMin, std::min(kBucketShift, sh));
+        uint64_t b;
+        std::memcpy(&b, &span[0], 8);
+        const int64_t base = (int64_t)(b >> sh) - 512;
+        dp_full.bucket_shift = sh;
+        dp_full.bucket_base = (uint32_t)std::max<int64_t>(0, base);
+        dp.bucket_shift = dp_full.bucket_shift;
+        dp.bucket_base = dp_full.bucket_base;
+        keep = 3;
+      }
+    }
+    k_init<<<1, 256, 0, st>>>(dp, keep);
     CK(cudaGetLastError());
     launches++;
+    if (keep == 3) {
+      k_rebucket<<<std::max(1, std::min(4 * nsm, (ncand0 + 255) / 256)), 256, 0, st>>>(dp, ncand0);
+      CK(cudaGetLastError());
+      launches++;
+    }
     if (pass == 2 && dp.want_pareto) {
       k_reseed<<<1, 1024, 0, st>>>(dp, (CandRec *)dp.out);
       CK(cudaGetLastError());

@@ -101,7 +101,9 @@ struct Thr {
 // exact makespan T (unnormalised, float, rounded down), eh = fp32 E/E_seq.
 // Buckets of a float coincide with buckets of the same value as a double.
 __device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParams &p, float tlb, float eh) {
-  const int b = (int)((__float_as_uint(tlb) >> 16) + (896u << 7)) - (int)p.bucket_base;
+  // bits64(x) >> s == (bits32(x) >> (s - 29)) + (896 << (52 - s)) for a float x, s >= 29
+  const int b = (int)((__float_as_uint(tlb) >> (p.bucket_shift - 29)) + (896u << (52 - p.bucket_shift))) -
+                (int)p.bucket_base;
   const int j = b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b);
   const unsigned int eb = __float_as_uint(eh);
   if (eb > s.pm[j]) return true;

@@ -194,7 +194,7 @@ class Scheduler:
                                  C.c_size_t(ws.numel()), C.c_void_p(st)), "sched_stage")
 
     def search(self, q, workspace=None, stream=None, pareto_cap=1 << 16, allow_infeasible=True,
-               **kw) -> SearchResult:
+               allow_capacity=False, **kw) -> SearchResult:
         import torch
         ws = workspace if workspace is not None else self.workspace(q, **kw)
         st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
@@ -206,7 +206,8 @@ class Scheduler:
         rc = lib().sched_search(self._h, C.byref(self.cquery(q, **kw)), C.c_void_p(ws.data_ptr()),
                                 C.c_size_t(ws.numel()), C.c_void_p(st), best, par, C.c_uint64(pareto_cap),
                                 C.byref(npar), C.byref(stats))
-        if rc != SCHED_OK and not (rc == SCHED_E_INFEASIBLE and allow_infeasible):
+        if rc != SCHED_OK and not (rc == SCHED_E_INFEASIBLE and allow_infeasible) and \
+                not (rc == SCHED_E_CAPACITY and allow_capacity):
             raise SchedError(rc, "sched_search")
         npv = min(npar.value, pareto_cap) if q.want_pareto else 0
         return SearchResult(rc, [best[w] for w in range(nw)], [par[k] for k in range(npv)],

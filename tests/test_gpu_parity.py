@@ -228,3 +228,26 @@ def test_tile_kernel_path(n, g, c, ws, seed):
     res = S.Scheduler(prof).search(q)
     assert res.stats["kernel_path"] == 1
     check(res, oracle.search(prof, q), q)
+
+
+def test_dense_local_front_window():
+    """A 3.3e12-configuration c4 window in the middle of the space whose local
+    Pareto front is dense inside the default staircase buckets (2^-7 relative
+    T width): before the seed-pass re-bucketing it flooded the candidate
+    buffer (SCHED_E_CAPACITY).  Must succeed, re-score exactly, and equal the
+    merge of its two halves."""
+    prof, q = config("c4")
+    lo, n = 100_000_000_000_000, 3 << 40
+    qw = q.with_range(lo, lo + n)
+    sch = S.Scheduler(prof)
+    res = sch.search(qw)
+    assert res.status == S.sched.SCHED_OK and res.stats["n_configs"] == n
+    assert res.stats["n_candidates"] < 1 << 20
+    for p in list(res.pareto) + list(res.best):
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
+        assert ok and (T, E) == (p.makespan_s, p.energy_j)
+    halves = [sch.search(q.with_range(lo, lo + n // 2)), sch.search(q.with_range(lo + n // 2, lo + n))]
+    mb, mp = S.merge([h.best for h in halves], [h.pareto for h in halves], len(q.weights))
+    assert [(b.index, b.score64) for b in mb] == [(b.index, b.score64) for b in res.best]
+    assert [(p.index, p.makespan_s, p.energy_j) for p in mp] == \
+        [(p.index, p.makespan_s, p.energy_j) for p in res.pareto]

@@ -21,12 +21,13 @@ if len(args) >= 3:
 sch = S.Scheduler(prof)
 for _ in range(reps):
     t0 = time.perf_counter()
-    r = sch.search(q)
+    r = sch.search(q, allow_capacity=True)
     dt = time.perf_counter() - t0
     st = r.stats
     print(json.dumps({"name": name, "kernel": os.environ.get("SCHED_KERNEL", "auto"), "wall_s": dt,
                       "search_ms": st["search_ms"], "configs": st["n_configs"],
                       "configs_per_s": st["n_configs"] / (st["search_ms"] / 1e3),
-                      "path": st["kernel_path"], "refined": st["n_refined"], "feasible": st["n_feasible"],
+                      "path": st["kernel_path"], "status": r.status, "passes": st["passes"], "cand": st["n_candidates"],
+                      "refined": st["n_refined"], "feasible": st["n_feasible"],
                       "best": [(b.index, b.score64) for b in r.best],
                       "pareto": [(p.index, p.makespan_s, p.energy_j) for p in r.pareto]}))
