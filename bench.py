@@ -30,7 +30,7 @@ METRIC = "configurations scored/sec (whole box) at 1/2/4/8 B200; time-to-optimal
 UNIT = "configs/s"
 SLICES = 64
 CHUNK_LOG2 = 22
-OPS_PER_CONFIG = 6   # T max, E add, 2 proxy mults, 2 min-reductions (c4)
+OPS_PER_CONFIG = 4   # T max, E add, 2 min-reductions (c4 tile kernel, per configuration)
 SMS = 148
 LANES_PER_SM_CLK = 4 * 32   # 4 SMSPs x 32 lanes issue slots per clock
 

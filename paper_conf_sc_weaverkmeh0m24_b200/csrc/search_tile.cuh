@@ -121,15 +121,17 @@ __device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParam
 // line (slow path).  Returns 1 if it issued a refine.
 template <class WS>
 __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, const Stair &stair,
-                                         const WarpPart &wp, const float *thr, BestRec *lb, u64 idx,
+                                         const WarpPart &wp, float *thr, BestRec *lb, u64 idx,
                                          const int *dig, float T, float E, double T64) {
   unsigned need = 0;
   if constexpr (WS::N > 0) {
     float q[WS::N];
     WS::q(T, E, q);
 #pragma unroll
-    for (int s = 0; s < WS::N; s++)
+    for (int s = 0; s < WS::N; s++) {
       if (q[s] <= fminf(thr[s], q[s]) * p.mul[p.ws_perm[s]]) need |= 1u << s;
+      thr[s] = fminf(thr[s], q[s]);
+    }
   }
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
@@ -197,7 +199,7 @@ __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, c
 // per-configuration checks.
 template <class WS>
 __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, const Stair &stair,
-                                      const WarpPart &wp, const float *thr, BestRec *lb, uint32_t vt, float Tp,
+                                      const WarpPart &wp, float *thr, BestRec *lb, uint32_t vt, float Tp,
                                       float Ep, bool arg_hit) {
   const int k = wp.cfg.k;
   int dig[kTileMaxG];
@@ -311,9 +313,12 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     bool hit = false;
     float cE;
     if constexpr (WS::N > 0) {
-      float mq[WS::N];
-#pragma unroll
-      for (int s = 0; s < WS::N; s++) mq[s] = __int_as_float(0x7f800000);
+      // every configuration's (T, E), min-reduced over the tile: the tile's
+      // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
+      // corner's proxies bound every configuration's from below (a tile
+      // whose corner misses every threshold holds no candidate); a tile that
+      // is not cleared is re-checked configuration by configuration.
+      float mT = __int_as_float(0x7f800000), mE = mT;
 #pragma unroll
       for (int a = 0; a < 4; a++) {
         const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
@@ -323,20 +328,16 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
 #pragma unroll
           for (int c = 0; c < 4; c++) {
             const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
-            float q[WS::N];
-            WS::q(T, E, q);
-#pragma unroll
-            for (int s = 0; s < WS::N; s++) mq[s] = fminf(mq[s], q[s]);
+            mT = fminf(mT, T);
+            mE = fminf(mE, E);
           }
         }
       }
+      float mq[WS::N];
+      WS::q(mT, mE, mq);
 #pragma unroll
-      for (int s = 0; s < WS::N; s++) {
-        thr.v[s] = fminf(thr.v[s], mq[s]);
-        hit |= mq[s] <= thr.v[s] * p.mul[p.ws_perm[s]];
-      }
-      // min over the tile of the fp32 E above ((Ep + a) + b) + c is monotone in each term
-      cE = ((Ep + minAe) + minBe) + minCe;
+      for (int s = 0; s < WS::N; s++) hit |= mq[s] <= thr.v[s] * p.mul[p.ws_perm[s]];
+      cE = mE;
     } else {  // Pareto only: per-configuration E, min-reduced
       cE = __int_as_float(0x7f800000);
 #pragma unroll
@@ -357,6 +358,8 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
 #pragma unroll
       for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
       nref += tile_slow<WS>(tb, p, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+#pragma unroll
+      for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
     }
   }
   __syncwarp();
