@@ -95,6 +95,7 @@ struct WarpPart {
 template <class WS>
 struct Thr {
   float v[WS::N > 0 ? WS::N : 1];
+  float m[WS::N > 0 ? WS::N : 1];  // 1 + delta of the weight in slot s (registers: no indexed param loads)
 };
 
 // quick Pareto screen from fp32 values: tlb = certified lower bound of the
@@ -236,9 +237,12 @@ __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, cons
 }
 
 // exact min fp64 makespan over a tile (its corner), k >= 5
-static __device__ __noinline__ double tile_corner64(const WarpPart &wp, uint32_t vt, double minC64) {
+static __device__ __noinline__ double tile_corner64(const WarpPart &wp, uint32_t vt) {
   const int k = wp.cfg.k;
-  double t = minC64;
+  const int ga = (k - 3) * 4, gb = (k - 2) * 4, gc = (k - 1) * 4;
+  double t = fmax(fmax(fmin(fmin(wp.g64[gb], wp.g64[gb + 1]), fmin(wp.g64[gb + 2], wp.g64[gb + 3])),
+                       fmin(fmin(wp.g64[gc], wp.g64[gc + 1]), fmin(wp.g64[gc + 2], wp.g64[gc + 3]))),
+                  fmin(fmin(wp.g64[ga], wp.g64[ga + 1]), fmin(wp.g64[ga + 2], wp.g64[ga + 3])));
   for (int b = 0; b < k - 3; b++) t = fmax(t, wp.g64[b * 4 + ((int)(vt >> (2 * (k - 1 - b))) & 3)]);
   return t;
 }
@@ -285,15 +289,10 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     Ct[m] = wp.gt[gc + m];
     Ce[m] = wp.ge[gc + m];
   }
-  const float minTin = fmaxf(fmaxf(fminf(fminf(At[0], At[1]), fminf(At[2], At[3])),
-                                   fminf(fminf(Bt[0], Bt[1]), fminf(Bt[2], Bt[3]))),
-                             fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
-  const float minAe = fminf(fminf(Ae[0], Ae[1]), fminf(Ae[2], Ae[3]));
-  const float minBe = fminf(fminf(Be[0], Be[1]), fminf(Be[2], Be[3]));
-  const float minCe = fminf(fminf(Ce[0], Ce[1]), fminf(Ce[2], Ce[3]));
-  const double mc64 = fmax(fmax(fmin(fmin(wp.g64[gb], wp.g64[gb + 1]), fmin(wp.g64[gb + 2], wp.g64[gb + 3])),
-                                fmin(fmin(wp.g64[gc], wp.g64[gc + 1]), fmin(wp.g64[gc + 2], wp.g64[gc + 3]))),
-                           fmin(fmin(wp.g64[ga], wp.g64[ga + 1]), fmin(wp.g64[ga + 2], wp.g64[ga + 3])));
+  const float minTin = WS::N > 0 ? 0.f
+                                 : fmaxf(fmaxf(fminf(fminf(At[0], At[1]), fminf(At[2], At[3])),
+                                               fminf(fminf(Bt[0], Bt[1]), fminf(Bt[2], Bt[3]))),
+                                         fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
   int nref = 0;
   const uint32_t s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
   for (uint32_t st = s_lo; st <= s_hi; st++) {
@@ -311,7 +310,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
       continue;
     }
     bool hit = false;
-    float cE;
+    float cE, cT;
     if constexpr (WS::N > 0) {
       // every configuration's (T, E), min-reduced over the tile: the tile's
       // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
@@ -336,9 +335,11 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
       float mq[WS::N];
       WS::q(mT, mE, mq);
 #pragma unroll
-      for (int s = 0; s < WS::N; s++) hit |= mq[s] <= thr.v[s] * p.mul[p.ws_perm[s]];
+      for (int s = 0; s < WS::N; s++) hit |= mq[s] <= thr.v[s] * thr.m[s];
       cE = mE;
+      cT = mT;
     } else {  // Pareto only: per-configuration E, min-reduced
+      cT = fmaxf(Tp, minTin);
       cE = __int_as_float(0x7f800000);
 #pragma unroll
       for (int a = 0; a < 4; a++) {
@@ -352,8 +353,8 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
       }
     }
     bool par = false;
-    if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(fmaxf(Tp, minTin), p.tlb_scale_f), cE))
-      par = !stair_dominated(stair, p, tile_corner64(wp, vt, mc64), cE);
+    if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
+      par = !stair_dominated(stair, p, tile_corner64(wp, vt), cE);
     if (hit || par) {
 #pragma unroll
       for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
@@ -387,6 +388,7 @@ __global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {
     thr.v[s] = __int_as_float(0x7f800000);
+    thr.m[s] = s < WS::N ? p.mul[p.ws_perm[s]] : 1.f;
     best_init(lb[s]);
   }
   u64 ncfg = 0, nfeas = 0, stair_ver = 0;
