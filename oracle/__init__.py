@@ -236,15 +236,16 @@ def objective(tseq, eseq, T, E, a, b) -> float:
 
 
 def dp_certificate(prof, q, cap: int = 1 << 20):
-    """O3 (dpcert.c): exact Pareto-front values [(T, E)] (T ascending) of the
-    whole PER_GPU space and the exact optimum F per weight (max over the
-    front, canonical fp64).  Values only, no indices."""
-    assert q.scope == 1, "certificate covers PER_GPU scope"
+    """O3 (PER_GPU) / O4 (PER_CLIENT) in dpcert.c: exact Pareto-front values
+    [(T, E)] (T ascending) of the whole space and the exact optimum F per
+    weight (max over the front, canonical fp64).  Values only, no indices."""
+    assert getattr(q, "model", 0) == 0, "certificate covers the canonical model"
     pk = _Pack(prof, q)
     ot = (C.c_double * cap)()
     oe = (C.c_double * cap)()
     lev = (C.c_int * len(pk.lev_idx))(*pk.lev_idx)
-    nf = lib().oracle_dpcert(C.byref(pk.P), q.n, q.g, min(q.c, q.n), len(q.levels), lev, ot, oe, cap)
+    fn = lib().oracle_dpcert if q.scope == 1 else lib().oracle_dpcert_client   # O3 / O4
+    nf = fn(C.byref(pk.P), q.n, q.g, min(q.c, q.n), len(q.levels), lev, ot, oe, cap)
     if nf < 0:
         raise RuntimeError("certificate capacity / size")
     front = [(ot[i], oe[i]) for i in range(nf)]

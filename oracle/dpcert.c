@@ -167,3 +167,120 @@ int oracle_dpcert(const or_profile *P0, int n, int g, int c, int L, const int *l
   free(gok);
   return nout;
 }
+
+/*
+ * O4: the same certificate for PER_CLIENT level scope (every client its own
+ * level, the literal reading of BASELINE.json's "per-client
+ * active-thread percentage").  A group's tuple now depends on its members'
+ * level vector: for every feasible group B the Pareto front PF(B) of
+ * (T_B, E_B) over all L^|B| level vectors is enumerated (plain loops,
+ * canonical order of enum.c), then the block-order DP of oracle_dpcert runs
+ * over those fronts.  Pruning dominated level vectors of a group is exact for
+ * the same reason as above (max and + are monotone under rounding).
+ */
+static int group_tuple_client(const or_profile *P, unsigned B, const int *pl, double *Tg_out,
+                              double *Eg_out) {
+  const int lp = P->lp, n = P->n;
+  long long M = 0;
+  for (int i = 0; i < n; i++) if (B >> i & 1) M += P->mem[i];
+  if (M > (long long)P->mem_cap) return 0;
+  double U = 0.0, Bw = 0.0;
+  for (int i = 0; i < n; i++) if (B >> i & 1) {
+    U = U + (double)P->u[i * lp + pl[i]];
+    Bw = Bw + (double)P->bw[i * lp + pl[i]];
+  }
+  double c = 1.0;
+  if (U > c) c = U;
+  if (Bw > c) c = Bw;
+  double Tg = 0.0;
+  for (int i = 0; i < n; i++) if (B >> i & 1) {
+    double sigma = 1.0;
+    for (int j = 0; j < n; j++) if ((B >> j & 1) && j != i)
+      sigma = sigma + (double)P->d[((size_t)(i * lp + pl[i]) * P->n + j) * lp + pl[j]];
+    double tau = ((double)P->t[i * lp + pl[i]] * sigma) * c;
+    if (tau > Tg) Tg = tau;
+  }
+  const double ps = (double)P->ps;
+  double D = 0.0;
+  for (int i = 0; i < n; i++) if (B >> i & 1)
+    D = D + ((double)P->p[i * lp + pl[i]] - ps) * (double)P->t[i * lp + pl[i]];
+  *Tg_out = Tg;
+  *Eg_out = ps * Tg + D;
+  return 1;
+}
+
+int oracle_dpcert_client(const or_profile *P0, int n, int g, int c, int L, const int *lev,
+                         double *out_t, double *out_e, int out_cap) {
+  if (n < 1 || n > 14) return -1;
+  or_profile Pv = *P0;
+  const or_profile *P = &Pv;
+  const unsigned full = (1u << n) - 1;
+  const size_t NS = (size_t)1 << n;
+  flist *PF = calloc(NS, sizeof(flist));   /* per-group front over level vectors */
+  for (unsigned B = 1; B <= full; B++) {
+    const int s = __builtin_popcount(B);
+    if (s > c) continue;
+    int mem[32], pl[64];
+    int m = 0;
+    for (int i = 0; i < n; i++) if (B >> i & 1) mem[m++] = i;
+    long long nv = 1;
+    for (int k = 0; k < s; k++) nv *= L;
+    for (long long v = 0; v < nv; v++) {
+      long long x = v;
+      for (int k = s - 1; k >= 0; k--) { pl[mem[k]] = lev[x % L]; x /= L; }
+      double Tg, Eg;
+      if (!group_tuple_client(P, B, pl, &Tg, &Eg)) break;   /* memory: same for every vector */
+      push(&PF[B], Tg, Eg);
+    }
+    prune(&PF[B]);
+  }
+  flist *F = calloc(NS * (size_t)(g + 1), sizeof(flist));
+  push(&F[0], 0.0, 0.0);
+  for (unsigned S = 0; S < full; S++) {
+    const unsigned rest = full & ~S;
+    const unsigned low = rest & (0u - rest);
+    const unsigned others = rest & ~low;
+    for (int k = 0; k < g; k++) {
+      flist *f = &F[(size_t)S * (g + 1) + k];
+      if (f->n == 0) continue;
+      prune(f);
+      unsigned sub = others;
+      for (;;) {
+        const unsigned B = low | sub;
+        const flist *pb = &PF[B];
+        if (pb->n) {
+          flist *to = &F[(size_t)(S | B) * (g + 1) + k + 1];
+          for (int q = 0; q < pb->n; q++) {
+            const double tb = pb->p[q].t, eb = pb->p[q].e;
+            for (int i = 0; i < f->n; i++) {
+              const double T = f->p[i].t > tb ? f->p[i].t : tb;
+              push(to, T, f->p[i].e + eb);
+            }
+          }
+        }
+        if (sub == 0) break;
+        sub = (sub - 1) & others;
+      }
+      free(f->p);
+      f->p = 0;
+      f->n = f->cap = 0;
+    }
+  }
+  flist fin = {0, 0, 0, 0};
+  for (int k = 1; k <= g; k++) {
+    flist *f = &F[(size_t)full * (g + 1) + k];
+    for (int i = 0; i < f->n; i++) push(&fin, f->p[i].t, f->p[i].e);
+    free(f->p);
+  }
+  prune(&fin);
+  int nout = fin.n;
+  if (nout <= out_cap)
+    for (int i = 0; i < nout; i++) { out_t[i] = fin.p[i].t; out_e[i] = fin.p[i].e; }
+  else
+    nout = -1;
+  free(fin.p);
+  free(F);
+  for (size_t B = 0; B < NS; B++) free(PF[B].p);
+  free(PF);
+  return nout;
+}

@@ -43,3 +43,22 @@ def test_golden_certificates_reproduce(name):
     cert = oracle.dp_certificate(prof, q)
     assert [[t.hex(), e.hex()] for t, e in cert["front"]] == g["front_T_E"]
     assert [b.hex() for b in cert["best"]] == g["best_score64"]
+
+
+@pytest.mark.parametrize("n,g,c,levels,seed", [
+    (5, 2, 3, (25, 50, 75, 100), 700), (6, 3, 3, (50, 100), 701), (7, 3, 7, (25, 50, 75, 100), 702),
+    (6, 4, 2, (50, 100), 703), (5, 5, 5, (25, 50, 75, 100), 704), (6, 6, 6, (25, 50, 75, 100), 706),
+    (8, 3, 3, (50, 100), 707),
+])
+def test_client_certificate_equals_enumeration(n, g, c, levels, seed):
+    """O4 (PER_CLIENT subset DP over per-group level-vector fronts) == O1 full
+    enumeration: front values and every weight's optimum, bitwise.  Catches:
+    a level-vector order or member-level mix-up in the per-client group tuple,
+    a dropped level vector, or pruning a vector that reaches the front."""
+    from synth import PER_CLIENT
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, levels, PER_CLIENT, W, True)
+    r = oracle.search(prof, q)
+    cert = oracle.dp_certificate(prof, q)
+    assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
+    assert [b[1] if b else None for b in r["best"]] == cert["best"]
