@@ -141,13 +141,25 @@ typedef struct {
   double t_seq_s, e_seq_j;      /* sequential baselines */
   float search_ms;              /* device time of the search kernel(s) (CUDA events) */
   float total_ms;               /* device time of the whole call on the stream */
-  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile kernel, 2 L=1 pair kernel, 3 L=1 suffix kernel */
+  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile, 2 L=1 pair, 3 L=1 suffix, 4 subset-DP front */
   int32_t grid_ctas;            /* persistent CTAs launched by the search kernel */
   int32_t kernel_launches;      /* kernels this call launched (init, search pass(es), finalize) */
   int32_t passes;               /* search passes (2 = re-run after candidate overflow) */
   uint64_t h2d_bytes;           /* host->device bytes this call copied (staged tables) */
   uint64_t d2h_bytes;           /* device->host bytes this call copied (counters, picks) */
 } sched_stats;
+
+/* One point of the exact front computed by sched_front_dp, with one witness
+ * configuration (no index: the literal per-client spaces exceed 2^64). */
+typedef struct {
+  double makespan_s, energy_j;  /* exact canonical fp64 T, E (bitwise the oracle's) */
+  double x64, y64;              /* X = T_seq/T, Y = E_seq/E */
+  double score64;               /* best[w]: F_w = X^a Y^b; front points: X */
+  int32_t n_groups;
+  int8_t group_of[SCHED_MAX_WORKFLOWS];  /* witness: RGS (block order) */
+  int8_t level_of[SCHED_MAX_WORKFLOWS];  /* witness: searched-level digit of each workflow */
+  int32_t valid;
+} sched_dp_point;
 
 typedef struct sched_handle sched_handle;
 
@@ -203,6 +215,24 @@ int sched_rank(const sched_query *q, const int8_t *group_of, const int8_t *level
  * with W == 0 score64 = X).  out->valid = 0 if memory-infeasible.  Host only. */
 int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int32_t w,
                 sched_pick *out);
+
+/* Exact Pareto front and per-weight optimum of the WHOLE space of the query
+ * by a subset dynamic program on the device (dp_front.cu):
+ * for every feasible group the Pareto front of its (T_g, E_g) over its level
+ * vectors, then the block-order DP over workflow subsets.  Reaches spaces
+ * that cannot be enumerated, e.g. the literal per-client c4 (16 workflows,
+ * 8 GPUs, 4 levels per client: 4.05e19 configurations).  Requires
+ * 2 <= n <= 16, L^max_clients <= 2^32 (PER_CLIENT), no SCHED_MODEL_COUNT_IDLE;
+ * the index window and shard fields must be the defaults (whole space, one
+ * shard).  front[front_cap] is ordered by X descending (T ascending), one
+ * witness configuration per distinct (T, E); best[W] is the max F_w over the
+ * front (ties: the first in that order; not necessarily the lowest index).
+ * Errors: INVALID, TOO_LARGE, WORKSPACE, CUDA, CAPACITY (an internal front
+ * overflowed, or *n_front > front_cap), INFEASIBLE (empty front), NODEVICE. */
+int sched_dp_workspace_size(const sched_handle *h, const sched_query *q, size_t *bytes);
+int sched_front_dp(sched_handle *h, const sched_query *q, void *d_workspace, size_t ws_bytes,
+                   void *cuda_stream, sched_dp_point *best, sched_dp_point *front, uint64_t front_cap,
+                   uint64_t *n_front, sched_stats *stats);
 
 /* The paper's rule-based co-scheduling heuristic (reading
  * R25 in DESIGN.md), for measuring its optimality gap against the exhaustive

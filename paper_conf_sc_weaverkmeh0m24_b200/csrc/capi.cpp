@@ -52,6 +52,25 @@ int resolve(sched_handle *h, const sched_query *qin, Query *q, const Space **sp)
   return SCHED_OK;
 }
 
+// query for the subset-DP front: shape + profile checks, whole space, one
+// shard; no DP count table (the literal per-client spaces exceed 2^63)
+int resolve_dp(sched_handle *h, const sched_query *qin, Query *q, std::vector<unsigned char> *blob, DevParams *dp) {
+  int st = resolve_query_shape(qin, h->P.lp, q);
+  if (st) return st;
+  if (q->n > h->P.n) return SCHED_E_INVALID;
+  if ((q->model & SCHED_MODEL_POWER_CAP) && !(q->pcap > h->P.ps)) return SCHED_E_INVALID;
+  if (q->lo != 0 || (q->hi != 0 && q->hi != UINT64_MAX) || q->count != 1) return SCHED_E_INVALID;
+  q->lo = 0;
+  q->hi = 0;
+  Space empty;
+  empty.n = q->n;
+  empty.g = q->g;
+  empty.c = q->c;
+  empty.L = q->L;
+  empty.scope = q->scope;
+  return build_stage(h->P, *q, empty, blob, dp);
+}
+
 int need_device() {
   int n = 0;
   if (cudaGetDeviceCount(&n) != cudaSuccess || n < 1) {
@@ -351,6 +370,81 @@ int sched_score(const sched_handle *hc, const sched_query *qin, uint64_t index, 
   out->y64 = es / E;
   const int ea = q.nw ? q.wa[w] : 1, eb = q.nw ? q.wb[w] : 0;
   out->score64 = host_objective(ts, es, T, E, ea, eb);
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_dp_workspace_size(const sched_handle *hc, const sched_query *qin, size_t *bytes) {
+  GUARD_BEGIN
+  if (!hc || !bytes) return SCHED_E_INVALID;
+  sched_handle *h = const_cast<sched_handle *>(hc);
+  Query q;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  int st = resolve_dp(h, qin, &q, &blob, &dp);
+  if (st) return st;
+  return dp_front_workspace(h->P, q, dp, bytes);
+  GUARD_END
+}
+
+int sched_front_dp(sched_handle *h, const sched_query *qin, void *ws, size_t ws_bytes, void *stream,
+                   sched_dp_point *best, sched_dp_point *front, uint64_t front_cap, uint64_t *n_front,
+                   sched_stats *stats) {
+  GUARD_BEGIN
+  if (!h || !ws || !n_front || (front_cap > 0 && !front)) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  Query q;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = resolve_dp(h, qin, &q, &blob, &dp);
+  if (st) return st;
+  if (q.nw > 0 && !best) return SCHED_E_INVALID;
+  std::vector<DpPoint> pts;
+  int bpos[kMaxW];
+  float ms = 0.f;
+  int launches = 0;
+  st = dp_front_run(h->P, q, dp, blob, ws, ws_bytes, stream, &pts, bpos, &ms, &launches);
+  if (st) return st;
+  double ts, es;
+  host_constants(h->P, q, &ts, &es);
+  auto fill = [&](const DpPoint &d, double score, sched_dp_point *o) {
+    std::memset(o, 0, sizeof *o);
+    o->valid = 1;
+    o->makespan_s = d.t;
+    o->energy_j = d.e;
+    o->x64 = ts / d.t;
+    o->y64 = es / d.e;
+    o->score64 = score;
+    o->n_groups = d.k;
+    for (int i = 0; i < q.n; i++) {
+      o->group_of[i] = d.group_of[i];
+      o->level_of[i] = d.level_of[i];
+    }
+  };
+  for (int w = 0; w < q.nw; w++) {
+    if (pts.empty() || bpos[w] < 0) {
+      std::memset(&best[w], 0, sizeof best[w]);
+      continue;
+    }
+    const DpPoint &d = pts[bpos[w]];
+    fill(d, host_objective(ts, es, d.t, d.e, q.wa[w], q.wb[w]), &best[w]);
+  }
+  *n_front = pts.size();
+  if (pts.size() <= front_cap)
+    for (size_t i = 0; i < pts.size(); i++) fill(pts[i], ts / pts[i].t, &front[i]);
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->t_seq_s = ts;
+    stats->e_seq_j = es;
+    stats->search_ms = ms;
+    stats->total_ms = ms;
+    stats->kernel_path = 4;
+    stats->kernel_launches = launches;
+    stats->h2d_bytes = blob.size();
+  }
+  if (pts.empty()) return SCHED_E_INFEASIBLE;
+  if (pts.size() > front_cap) return SCHED_E_CAPACITY;
   return SCHED_OK;
   GUARD_END
 }

@@ -1,0 +1,634 @@
+// dp_front.cu -- exact Pareto front and optimum by a subset DP on the device
+// (SURVEY 8(f) N1): spaces too large to enumerate, in particular the literal
+// per-client reading of c4 (BASELINE.json "per-client active-thread
+// percentage": 16 workflows x 8 GPUs x 4 levels per CLIENT = 4.05e19
+// configurations, more than 2^64).
+//
+// A configuration is a sequence of groups in block order (group j holds the
+// smallest workflow not in groups 0..j-1) with a level vector per group;
+// T = max_g T_g and E = ((0 + E_0) + E_1) + ... in that order (DESIGN.md
+// section 2).  Both maps are monotone under IEEE rounding, so dominated
+// partial results can be dropped without losing a final Pareto point:
+//   phase 1 (k_pf_items, k_pf_merge): for every feasible group B the Pareto
+//     front PF(B) of its exact canonical fp64 (T_B, E_B) over all level
+//     vectors (L^|B| PER_CLIENT, L PER_GPU);
+//   phase 2 (k_dp_level, one launch per |S|): Front[S][k] = Pareto front of
+//     { (max(T, T_b), E + E_b) : (T, E) in Front[S \ B][k-1], b in PF(B) }
+//     over the last groups B of S (B holds an element below min(~S));
+//   phase 3 (k_dp_final): the front of the whole set over k <= G, the best
+//     point per weight (max F = X^a Y^b, first in T order on ties) and a
+//     witness configuration per point traced through back-pointers.
+// Everything is exact fp64 in the canonical order; the result equals the
+// oracle's O4/O3 certificate (oracle/dpcert.c) bitwise.  Values and one
+// witness per point; ties between distinct configurations of equal (T, E)
+// are not resolved to the lowest index (the literal space has no u64 index).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <vector>
+
+#include "device_common.cuh"
+
+namespace sched {
+
+constexpr int kLF = 16;     // lane-local front capacity (phase 1)
+constexpr int kOF = 16;     // per work item / per group front capacity
+constexpr int kFM = 32;     // per DP state front capacity
+constexpr int kItemLog2 = 18;  // level vectors per phase-1 work item
+
+struct PPt {  // a group tuple: exact (T_B, E_B) of level vector v
+  double t, e;
+  uint32_t v, pad;
+};
+
+struct DPt {  // a DP state point and its back-pointer
+  double t, e;
+  uint32_t B;     // last group
+  uint8_t i, q;   // point in Front[S \ B][k-1] (0xff: S == B), point in PF(B)
+  uint16_t pad;
+};
+
+enum { kDpItem = 0, kDpErr = 1, kDpN = 4 };
+
+struct DpParams {
+  DevParams p;                 // tables (blob), scope, L, G, C, model, ps
+  int n, ns, nfull;            // workflows, subsets, n_items (phase 1)
+  const uint32_t *smask;       // [ns] subsets (ascending)
+  const unsigned long long *ioff;  // [ns + 1] item offsets
+  const int *sid;              // [2^n] subset id of a mask, -1 if none
+  PPt *items;                  // [n_items][kOF]
+  int *icnt;                   // [n_items]
+  PPt *pf;                     // [ns][kOF]
+  int *pfcnt;                  // [ns]
+  DPt *fr;                     // [2^(n-1)][G+1][kFM] (states contain workflow 0)
+  int *frcnt;                  // [2^(n-1)][G+1]
+  unsigned long long *ctr;     // [kDpN]
+};
+
+__device__ __forceinline__ bool dom(double t1, double e1, double t2, double e2) {  // (1) dominates (2)
+  return t1 <= t2 && e1 <= e2 && (t1 < t2 || e1 < e2);
+}
+
+// insert into a small front (local memory); returns false on overflow
+template <int CAP, class P>
+__device__ __forceinline__ bool front_insert(P *f, int &n, const P &x) {
+  for (int j = 0; j < n; j++)
+    if (f[j].t <= x.t && f[j].e <= x.e) return true;  // dominated or equal: keep the first
+  int w = 0;
+  for (int j = 0; j < n; j++)
+    if (!(x.t <= f[j].t && x.e <= f[j].e)) f[w++] = f[j];
+  n = w;
+  if (n >= CAP) return false;
+  f[n++] = x;
+  return true;
+}
+
+// exact canonical fp64 (T_B, E_B) of group B with per-member level digits
+// lev[i] (digit of workflow i); false if infeasible (R27)
+__device__ __forceinline__ bool group64(const Tables &tb, const DevParams &p, uint32_t B, const int *lev,
+                                        double &Tout, double &Eout) {
+  const double ps = p.ps;
+  double U = 0.0, Bw = 0.0;
+  for (uint32_t m = B; m; m &= m - 1) {
+    const int i = __ffs(m) - 1, r = i * p.L + lev[i];
+    U = __dadd_rn(U, (double)tb.u[r]);
+    Bw = __dadd_rn(Bw, (double)tb.bw[r]);
+  }
+  if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (U > 1.0 || Bw > 1.0)) return false;
+  double c = 1.0;
+  if (U > c) c = U;
+  if (Bw > c) c = Bw;
+  double Tg = 0.0;
+  for (uint32_t m = B; m; m &= m - 1) {
+    const int i = __ffs(m) - 1, ri = i * p.L + lev[i];
+    double sigma = 1.0;
+    for (uint32_t m2 = B & ~(1u << i); m2; m2 &= m2 - 1) {
+      const int j = __ffs(m2) - 1;
+      sigma = __dadd_rn(sigma, (double)tb.d[ri * p.ds + j * p.L + lev[j]]);
+    }
+    const double tau = __dmul_rn(__dmul_rn((double)tb.traw[ri], sigma), c);
+    if (tau > Tg) Tg = tau;
+  }
+  double D = 0.0;
+  for (uint32_t m = B; m; m &= m - 1) {
+    const int i = __ffs(m) - 1, r = i * p.L + lev[i];
+    D = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]));
+  }
+  if (p.model & SCHED_MODEL_POWER_CAP) {
+    const double tcap = __ddiv_rn(D, p.capd);
+    if (tcap > Tg) Tg = tcap;
+  }
+  Tout = Tg;
+  Eout = __dadd_rn(__dmul_rn(ps, Tg), D);
+  return true;
+}
+
+// level digits of vector v for group B: PER_CLIENT the members' digits in
+// base L, most significant = lowest member; PER_GPU one digit for all
+__device__ __forceinline__ void decode_vec(const DevParams &p, uint32_t B, uint32_t v, int *lev) {
+  if (p.scope == SCHED_PER_GPU) {
+    for (uint32_t m = B; m; m &= m - 1) lev[__ffs(m) - 1] = (int)v;
+    return;
+  }
+  uint32_t x = v;
+  for (int i = 31; i >= 0; i--)
+    if (B >> i & 1u) {
+      lev[i] = (int)(x % (uint32_t)p.L);
+      x /= (uint32_t)p.L;
+    }
+}
+
+// phase 1a: work item = (group, 2^kItemLog2 level vectors); one warp per item
+__global__ void __launch_bounds__(256) k_pf_items(const DpParams dp) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  stage_blob(sm, dp.p);
+  const Tables tb = tables_at(sm, dp.p);
+  const int lane = threadIdx.x & 31;
+  for (;;) {
+    unsigned long long it = 0;
+    if (lane == 0) it = atomicAdd(dp.ctr + kDpItem, 1ull);
+    it = __shfl_sync(0xffffffffu, it, 0);
+    if (it >= (unsigned long long)dp.nfull) break;
+    int lo = 0, hi = dp.ns - 1;  // subset of the item: ioff[s] <= it < ioff[s+1]
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (dp.ioff[mid] <= it) lo = mid;
+      else hi = mid - 1;
+    }
+    const uint32_t B = dp.smask[lo];
+    const int s = __popc(B);
+    uint64_t nv = dp.p.scope == SCHED_PER_GPU ? (uint64_t)dp.p.L : 1ull;
+    if (dp.p.scope != SCHED_PER_GPU)
+      for (int k = 0; k < s; k++) nv *= (uint64_t)dp.p.L;
+    const uint64_t v0 = (it - dp.ioff[lo]) << kItemLog2;
+    const uint64_t v1 = v0 + (1ull << kItemLog2) < nv ? v0 + (1ull << kItemLog2) : nv;
+    PPt f[kLF];
+    int nf = 0;
+    bool ok = true;
+    int lev[kMaxN];
+    for (uint64_t v = v0 + lane; v < v1; v += 32) {
+      decode_vec(dp.p, B, (uint32_t)v, lev);
+      PPt x;
+      if (!group64(tb, dp.p, B, lev, x.t, x.e)) continue;
+      x.v = (uint32_t)v;
+      x.pad = 0;
+      ok &= front_insert<kLF>(f, nf, x);
+    }
+    if (!ok) atomicExch(dp.ctr + kDpErr, 1ull);
+    // warp merge: every lane keeps its points not dominated by another lane's
+    // (ties: the lower (lane, slot) wins), survivors compacted by ballot
+    PPt *out = dp.items + it * kOF;
+    int nout = 0;
+    for (int r = 0; r < kLF; r++) {  // round r: slot r of every lane
+      const bool has = r < nf;
+      if (!__any_sync(0xffffffffu, has)) break;
+      PPt x = has ? f[r] : PPt{0, 0, 0, 0};
+      bool keep = has;
+      for (int o = 0; o < 32; o++) {  // compare with every point of lane o
+        const int no = __shfl_sync(0xffffffffu, nf, o);
+        for (int q = 0; q < no; q++) {
+          PPt y;
+          y.t = __shfl_sync(0xffffffffu, f[min(q, kLF - 1)].t, o);
+          y.e = __shfl_sync(0xffffffffu, f[min(q, kLF - 1)].e, o);
+          if (keep && (dom(y.t, y.e, x.t, x.e) ||
+                       (y.t == x.t && y.e == x.e && (o < lane || (o == lane && q < r)))))
+            keep = false;
+        }
+      }
+      const unsigned bal = __ballot_sync(0xffffffffu, keep);
+      const int pos = nout + __popc(bal & ((1u << lane) - 1));
+      if (keep) {
+        if (pos < kOF) out[pos] = x;
+        else atomicExch(dp.ctr + kDpErr, 1ull);
+      }
+      nout += __popc(bal);
+    }
+    if (lane == 0) dp.icnt[it] = min(nout, kOF);
+  }
+}
+
+// phase 1b: PF(B) = front of the group's item fronts; one warp per group
+__global__ void __launch_bounds__(256) k_pf_merge(const DpParams dp) {
+  __shared__ PPt fs[8][kOF + 1];
+  __shared__ int fn[8];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  PPt *f = fs[warp];
+  for (int sb = blockIdx.x * 8 + warp; sb < dp.ns; sb += gridDim.x * 8) {
+    if (lane == 0) fn[warp] = 0;
+    __syncwarp();
+    const unsigned long long i0 = dp.ioff[sb], i1 = dp.ioff[sb + 1];
+    for (unsigned long long it = i0; it < i1; it++) {
+      const int c = dp.icnt[it];
+      for (int q0 = 0; q0 < c; q0 += 32) {  // a batch of up to 32 candidates, one per lane
+        const int q = q0 + lane;
+        PPt x = q < c ? dp.items[it * kOF + q] : PPt{0, 0, 0, 0};
+        bool keep = q < c;
+        const int n0 = fn[warp];
+        for (int j = 0; j < n0 && keep; j++)
+          if (f[j].t <= x.t && f[j].e <= x.e) keep = false;
+        unsigned bal = __ballot_sync(0xffffffffu, keep);
+        while (bal) {  // insert survivors in lane order
+          const int l = __ffs(bal) - 1;
+          bal &= bal - 1;
+          PPt y;
+          y.t = __shfl_sync(0xffffffffu, x.t, l);
+          y.e = __shfl_sync(0xffffffffu, x.e, l);
+          y.v = __shfl_sync(0xffffffffu, x.v, l);
+          y.pad = 0;
+          if (lane == 0) {
+            int n = fn[warp];
+            bool in = true;
+            for (int j = 0; j < n; j++)
+              if (f[j].t <= y.t && f[j].e <= y.e) in = false;
+            if (in) {
+              int w = 0;
+              for (int j = 0; j < n; j++)
+                if (!(y.t <= f[j].t && y.e <= f[j].e)) f[w++] = f[j];
+              if (w < kOF) f[w++] = y;
+              else atomicExch(dp.ctr + kDpErr, 1ull);
+              fn[warp] = w;
+            }
+          }
+          __syncwarp();
+        }
+      }
+    }
+    __syncwarp();
+    const int n = fn[warp];
+    for (int j = lane; j < n; j += 32) dp.pf[(size_t)sb * kOF + j] = f[j];
+    if (lane == 0) dp.pfcnt[sb] = n;
+    __syncwarp();
+  }
+}
+
+// phase 2: states S (containing workflow 0) with |S| = m; warp per (S, k)
+__global__ void __launch_bounds__(256) k_dp_level(const DpParams dp, int m, int nstates,
+                                                  const uint32_t *states) {
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int G = dp.p.g, C = dp.p.c;
+  const int wid = blockIdx.x * 8 + warp;
+  if (wid >= nstates * G) return;
+  const uint32_t S = states[wid / G];
+  const int k = wid % G + 1;  // groups in S
+  const uint32_t full = dp.n >= 32 ? 0xffffffffu : (1u << dp.n) - 1;
+  const uint32_t outside = full & ~S;
+  const int fmin = outside ? __ffs(outside) - 1 : dp.n;  // smallest workflow not in S
+  const uint32_t below = fmin >= 32 ? 0xffffffffu : (1u << fmin) - 1;  // B must meet these
+  DPt f[kFM];
+  int nf = 0;
+  bool ok = true;
+  const uint32_t nsub = 1u << m;
+  for (uint32_t x = 1 + lane; x < nsub; x += 32) {
+    uint32_t B = 0, xx = x;  // x-th subset of S (bit deposit)
+    for (uint32_t mm = S; mm && xx; mm &= mm - 1, xx >>= 1)
+      if (xx & 1u) B |= mm & (0u - mm);
+    if (!(B & below) || __popc(B) > C) continue;
+    const int sb = dp.sid[B];
+    if (sb < 0) continue;
+    const int npf = dp.pfcnt[sb];
+    if (!npf) continue;
+    const uint32_t R = S & ~B;
+    if (R == 0) {
+      if (k != 1) continue;
+      for (int q = 0; q < npf; q++) {
+        const PPt b = dp.pf[(size_t)sb * kOF + q];
+        DPt y{b.t, b.e, B, 0xff, (uint8_t)q, 0};
+        ok &= front_insert<kFM>(f, nf, y);
+      }
+      continue;
+    }
+    if (k == 1 || !(R & 1u)) continue;
+    const size_t src = ((size_t)(R >> 1) * (G + 1) + (k - 1));
+    const int nr = dp.frcnt[src];
+    for (int i = 0; i < nr; i++) {
+      const DPt a = dp.fr[src * kFM + i];
+      for (int q = 0; q < npf; q++) {
+        const PPt b = dp.pf[(size_t)sb * kOF + q];
+        DPt y{a.t > b.t ? a.t : b.t, __dadd_rn(a.e, b.e), B, (uint8_t)i, (uint8_t)q, 0};
+        ok &= front_insert<kFM>(f, nf, y);
+      }
+    }
+  }
+  if (!ok) atomicExch(dp.ctr + kDpErr, 1ull);
+  // warp merge (ties: lower (lane, slot) wins), write the state's front
+  const size_t dst = (size_t)(S >> 1) * (G + 1) + k;
+  int nout = 0;
+  for (int r = 0; r < kFM; r++) {
+    const bool has = r < nf;
+    if (!__any_sync(0xffffffffu, has)) break;
+    DPt x = has ? f[r] : DPt{0, 0, 0, 0, 0, 0};
+    bool keep = has;
+    for (int o = 0; o < 32; o++) {
+      const int no = __shfl_sync(0xffffffffu, nf, o);
+      for (int q = 0; q < no; q++) {
+        const double yt = __shfl_sync(0xffffffffu, f[min(q, kFM - 1)].t, o);
+        const double ye = __shfl_sync(0xffffffffu, f[min(q, kFM - 1)].e, o);
+        if (keep && (dom(yt, ye, x.t, x.e) || (yt == x.t && ye == x.e && (o < lane || (o == lane && q < r)))))
+          keep = false;
+      }
+    }
+    const unsigned bal = __ballot_sync(0xffffffffu, keep);
+    const int pos = nout + __popc(bal & ((1u << lane) - 1));
+    if (keep) {
+      if (pos < kFM) dp.fr[dst * kFM + pos] = x;
+      else atomicExch(dp.ctr + kDpErr, 1ull);
+    }
+    nout += __popc(bal);
+  }
+  if (lane == 0) dp.frcnt[dst] = min(nout, kFM);
+}
+
+// phase 3: front of the whole set over k = 1..G (ordered by T, then E) with
+// witness configurations (group masks in block order + level vectors)
+struct DpOut {
+  double t, e;
+  uint32_t groups[kMaxG];
+  uint32_t vecs[kMaxG];
+  int k;
+  int pad;
+};
+
+__global__ void k_dp_final(const DpParams dp, DpOut *out, int cap, int *nout, int *best) {
+  // single thread: at most G * kFM candidates
+  if (threadIdx.x || blockIdx.x) return;
+  const int G = dp.p.g;
+  const uint32_t full = dp.n >= 32 ? 0xffffffffu : (1u << dp.n) - 1;
+  int n = 0;
+  for (int k = 1; k <= G; k++) {
+    const size_t st = (size_t)(full >> 1) * (G + 1) + k;
+    for (int i = 0; i < dp.frcnt[st]; i++) {
+      const DPt x = dp.fr[st * kFM + i];
+      bool keep = true;
+      for (int k2 = 1; k2 <= G && keep; k2++) {
+        const size_t s2 = (size_t)(full >> 1) * (G + 1) + k2;
+        for (int j = 0; j < dp.frcnt[s2]; j++) {
+          const DPt y = dp.fr[s2 * kFM + j];
+          if (dom(y.t, y.e, x.t, x.e) || (y.t == x.t && y.e == x.e && (k2 < k || (k2 == k && j < i)))) {
+            keep = false;
+            break;
+          }
+        }
+      }
+      if (!keep) continue;
+      if (n < cap) {
+        DpOut &o = out[n];
+        o.t = x.t;
+        o.e = x.e;
+        // trace back through the states
+        uint32_t S = full;
+        int kk = k, pi = i, g = k - 1;
+        while (g >= 0) {
+          const DPt y = dp.fr[((size_t)(S >> 1) * (G + 1) + kk) * kFM + pi];
+          o.groups[g] = y.B;
+          o.vecs[g] = dp.pf[(size_t)dp.sid[y.B] * kOF + y.q].v;
+          S &= ~y.B;
+          kk--;
+          g--;
+          if (y.i == 0xff) break;
+          pi = y.i;
+        }
+        o.k = k;
+      }
+      n++;
+    }
+  }
+  // order by T ascending (then E): insertion sort on the output
+  const int m = n < cap ? n : cap;
+  for (int a = 1; a < m; a++) {
+    DpOut x = out[a];
+    int b = a - 1;
+    while (b >= 0 && (out[b].t > x.t || (out[b].t == x.t && out[b].e > x.e))) {
+      out[b + 1] = out[b];
+      b--;
+    }
+    out[b + 1] = x;
+  }
+  *nout = n;
+  // best point per weight: max F = X^a Y^b (fp64 canonical), first in T order on ties
+  for (int w = 0; w < dp.p.nw; w++) {
+    int bi = -1;
+    double bf = 0.0;
+    for (int a = 0; a < m; a++) {
+      const double F = objective64(dp.p, out[a].t, out[a].e, dp.p.wa[w], dp.p.wb[w]);
+      if (bi < 0 || F > bf) {
+        bi = a;
+        bf = F;
+      }
+    }
+    best[w] = bi;
+  }
+}
+
+// ------------------------------------------------------------------ host side
+namespace {
+struct DpLayout {
+  size_t ctr, blob, smask, ioff, sid, items, icnt, pf, pfcnt, fr, frcnt, states, out, nout, total;
+};
+
+DpLayout dp_layout(const DevParams &p, int n, int ns, uint64_t nitems, size_t nstates) {
+  DpLayout L;
+  size_t o = 0;
+  auto take = [&](size_t b) {
+    o = (o + 255) / 256 * 256;
+    const size_t r = o;
+    o += b;
+    return r;
+  };
+  L.ctr = take(8 * kDpN);
+  L.blob = take(p.blob_bytes);
+  L.smask = take(4 * (size_t)ns);
+  L.ioff = take(8 * ((size_t)ns + 1));
+  L.sid = take(4 * ((size_t)1 << n));
+  L.items = take(sizeof(PPt) * kOF * (size_t)nitems);
+  L.icnt = take(4 * (size_t)nitems);
+  L.pf = take(sizeof(PPt) * kOF * (size_t)ns);
+  L.pfcnt = take(4 * (size_t)ns);
+  L.fr = take(sizeof(DPt) * kFM * ((size_t)1 << (n - 1)) * (p.g + 1));
+  L.frcnt = take(4 * ((size_t)1 << (n - 1)) * (p.g + 1));
+  L.states = take(4 * nstates);
+  L.out = take(sizeof(DpOut) * (size_t)kFM * p.g);
+  L.nout = take(8 + 4 * kMaxW);
+  L.total = (o + 255) / 256 * 256;
+  return L;
+}
+
+// the feasible groups (|B| <= C, memory) and the phase-1 work items
+void dp_groups(const Profile &P, const Query &q, std::vector<uint32_t> *smask, std::vector<unsigned long long> *ioff,
+               std::vector<int> *sid) {
+  const int n = q.n;
+  sid->assign((size_t)1 << n, -1);
+  smask->clear();
+  ioff->assign(1, 0ull);
+  for (uint32_t B = 1; B < (1u << n); B++) {
+    const int s = __builtin_popcount(B);
+    if (s > q.c) continue;
+    long long M = 0;
+    for (int i = 0; i < n; i++)
+      if (B >> i & 1u) M += P.mem[i];
+    if (M > (long long)P.mem_cap) continue;
+    unsigned long long nv = 1;
+    if (q.scope == SCHED_PER_GPU) nv = (unsigned long long)q.L;
+    else
+      for (int k = 0; k < s; k++) nv *= (unsigned long long)q.L;
+    (*sid)[B] = (int)smask->size();
+    smask->push_back(B);
+    ioff->push_back(ioff->back() + ((nv + (1ull << kItemLog2) - 1) >> kItemLog2));
+  }
+}
+}  // namespace
+
+int dp_front_workspace(const Profile &P, const Query &q, const DevParams &dp, size_t *bytes) {
+  if (q.n < 2 || q.n > 16 || q.g > kMaxG || (q.model & SCHED_MODEL_COUNT_IDLE)) return SCHED_E_INVALID;
+  if (q.scope == SCHED_PER_CLIENT) {
+    double lg = 0.0;  // L^C must fit the 32-bit vector id
+    for (int k = 0; k < q.c; k++) lg += std::log2((double)q.L);
+    if (lg > 32.0) return SCHED_E_TOO_LARGE;
+  }
+  std::vector<uint32_t> smask;
+  std::vector<unsigned long long> ioff;
+  std::vector<int> sid;
+  dp_groups(P, q, &smask, &ioff, &sid);
+  const size_t nst = (size_t)1 << (q.n - 1);
+  *bytes = dp_layout(dp, q.n, (int)smask.size(), ioff.back(), nst).total;
+  return SCHED_OK;
+}
+
+#define CKD(x)                                  \
+  do {                                          \
+    cudaError_t e_ = (x);                       \
+    if (e_ != cudaSuccess) return SCHED_E_CUDA; \
+  } while (0)
+
+int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vector<unsigned char> &blob, void *d_ws,
+                 size_t ws_bytes, void *stream, std::vector<DpPoint> *front, int *best_pos, float *ms,
+                 int *launches) {
+  size_t need = 0;
+  int st = dp_front_workspace(P, q, p, &need);
+  if (st) return st;
+  if (ws_bytes < need || ((uintptr_t)d_ws & 255)) return SCHED_E_WORKSPACE;
+  std::vector<uint32_t> smask;
+  std::vector<unsigned long long> ioff;
+  std::vector<int> sid;
+  dp_groups(P, q, &smask, &ioff, &sid);
+  const int n = q.n, ns = (int)smask.size(), G = q.g;
+  // states containing workflow 0, by popcount
+  std::vector<std::vector<uint32_t>> lv(n + 1);
+  for (uint32_t S = 1; S < (1u << n); S += 2) lv[__builtin_popcount(S)].push_back(S);
+  const size_t nst = (size_t)1 << (n - 1);
+  const DpLayout L = dp_layout(p, n, ns, ioff.back(), nst);
+  unsigned char *ws = (unsigned char *)d_ws;
+  cudaStream_t s = (cudaStream_t)stream;
+  DpParams dp;
+  p.blob = ws + L.blob;
+  dp.p = p;
+  dp.n = n;
+  dp.ns = ns;
+  dp.nfull = (int)ioff.back();
+  dp.smask = (const uint32_t *)(ws + L.smask);
+  dp.ioff = (const unsigned long long *)(ws + L.ioff);
+  dp.sid = (const int *)(ws + L.sid);
+  dp.items = (PPt *)(ws + L.items);
+  dp.icnt = (int *)(ws + L.icnt);
+  dp.pf = (PPt *)(ws + L.pf);
+  dp.pfcnt = (int *)(ws + L.pfcnt);
+  dp.fr = (DPt *)(ws + L.fr);
+  dp.frcnt = (int *)(ws + L.frcnt);
+  dp.ctr = (unsigned long long *)(ws + L.ctr);
+  CKD(cudaMemsetAsync(ws + L.ctr, 0, 8 * kDpN, s));
+  CKD(cudaMemsetAsync(ws + L.frcnt, 0, 4 * nst * (G + 1), s));
+  CKD(cudaMemcpyAsync(ws + L.blob, blob.data(), blob.size(), cudaMemcpyHostToDevice, s));
+  CKD(cudaMemcpyAsync(ws + L.smask, smask.data(), 4 * smask.size(), cudaMemcpyHostToDevice, s));
+  CKD(cudaMemcpyAsync(ws + L.ioff, ioff.data(), 8 * ioff.size(), cudaMemcpyHostToDevice, s));
+  CKD(cudaMemcpyAsync(ws + L.sid, sid.data(), 4 * sid.size(), cudaMemcpyHostToDevice, s));
+  int dev = 0, nsm = 0;
+  CKD(cudaGetDevice(&dev));
+  CKD(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  cudaEvent_t e0, e1;
+  CKD(cudaEventCreate(&e0));
+  CKD(cudaEventCreate(&e1));
+  CKD(cudaEventRecord(e0, s));
+  int nl = 0;
+  const size_t smem = (p.blob_bytes + 15) & ~15u;
+  CKD(cudaFuncSetAttribute(k_pf_items, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  if (dp.nfull > 0) {
+    k_pf_items<<<nsm * 4, 256, smem, s>>>(dp);
+    CKD(cudaGetLastError());
+    nl++;
+    k_pf_merge<<<std::max(1, std::min(nsm * 8, (ns + 7) / 8)), 256, 0, s>>>(dp);
+    CKD(cudaGetLastError());
+    nl++;
+  }
+  // per-level state lists (uploaded once, consecutive)
+  std::vector<uint32_t> all;
+  std::vector<size_t> at(n + 1, 0);
+  for (int m = 1; m <= n; m++) {
+    at[m] = all.size();
+    all.insert(all.end(), lv[m].begin(), lv[m].end());
+  }
+  CKD(cudaMemcpyAsync(ws + L.states, all.data(), 4 * all.size(), cudaMemcpyHostToDevice, s));
+  for (int m = 1; m <= n; m++) {
+    const int nsts = (int)lv[m].size();
+    if (!nsts) continue;
+    const int warps = nsts * G;
+    k_dp_level<<<(warps + 7) / 8, 256, 0, s>>>(dp, m, nsts, (const uint32_t *)(ws + L.states) + at[m]);
+    CKD(cudaGetLastError());
+    nl++;
+  }
+  const int cap = kFM * G;
+  k_dp_final<<<1, 32, 0, s>>>(dp, (DpOut *)(ws + L.out), cap, (int *)(ws + L.nout), (int *)(ws + L.nout) + 2);
+  CKD(cudaGetLastError());
+  nl++;
+  CKD(cudaEventRecord(e1, s));
+  unsigned long long ctr[kDpN];
+  int hdr[2 + kMaxW];
+  CKD(cudaMemcpyAsync(ctr, ws + L.ctr, sizeof ctr, cudaMemcpyDeviceToHost, s));
+  CKD(cudaMemcpyAsync(hdr, ws + L.nout, sizeof hdr, cudaMemcpyDeviceToHost, s));
+  CKD(cudaStreamSynchronize(s));
+  const int nout = hdr[0];
+  for (int w = 0; w < q.nw; w++) best_pos[w] = hdr[2 + w];
+  std::vector<DpOut> outv((size_t)std::min(nout, cap));
+  if (!outv.empty()) {
+    CKD(cudaMemcpyAsync(outv.data(), ws + L.out, sizeof(DpOut) * outv.size(), cudaMemcpyDeviceToHost, s));
+    CKD(cudaStreamSynchronize(s));
+  }
+  CKD(cudaEventElapsedTime(ms, e0, e1));
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  *launches = nl;
+  if (ctr[kDpErr]) return SCHED_E_CAPACITY;
+  if (nout > cap) return SCHED_E_CAPACITY;
+  front->clear();
+  for (const DpOut &o : outv) {
+    DpPoint d;
+    std::memset(&d, 0, sizeof d);
+    d.t = o.t;
+    d.e = o.e;
+    d.k = o.k;
+    for (int g = 0; g < o.k; g++) {
+      const uint32_t B = o.groups[g];
+      std::vector<int> digits(n, 0);
+      uint32_t x = o.vecs[g];
+      if (q.scope == SCHED_PER_GPU) {
+        for (int i = 0; i < n; i++)
+          if (B >> i & 1u) digits[i] = (int)x;
+      } else {
+        for (int i = n - 1; i >= 0; i--)
+          if (B >> i & 1u) {
+            digits[i] = (int)(x % (uint32_t)q.L);
+            x /= (uint32_t)q.L;
+          }
+      }
+      for (int i = 0; i < n; i++)
+        if (B >> i & 1u) {
+          d.group_of[i] = (int8_t)g;
+          d.level_of[i] = (int8_t)digits[i];
+        }
+    }
+    front->push_back(d);
+  }
+  return SCHED_OK;
+}
+
+}  // namespace sched

@@ -166,6 +166,18 @@ int merge_picks(int n_ranks, int nw, const sched_pick *rank_best, const sched_pi
                 const uint64_t *rank_np, sched_pick *best, sched_pick *pareto, uint64_t cap,
                 uint64_t *np);
 
+// ---- subset-DP front (dp_front.cu) ----
+struct DpPoint {           // a front point with one witness configuration
+  double t, e;             // exact canonical fp64 T, E
+  int k;                   // groups
+  int8_t group_of[kMaxN];  // RGS (block order)
+  int8_t level_of[kMaxN];  // searched-level digit per workflow
+};
+int dp_front_workspace(const Profile &P, const Query &q, const DevParams &dp, size_t *bytes);
+int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vector<unsigned char> &blob, void *d_ws,
+                 size_t ws_bytes, void *stream, std::vector<DpPoint> *front, int *best_pos, float *ms,
+                 int *launches);
+
 // ---- device launchers (search.cu) ----
 struct LaunchInfo {
   int path, grid, launches, passes;

@@ -32,7 +32,7 @@ UINT64_MAX = (1 << 64) - 1
 
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
            "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score", "sched_heuristic",
-           "sched_strerror", "sched_version"]
+           "sched_strerror", "sched_version", "sched_dp_workspace_size", "sched_front_dp"]
 
 
 class SchedError(RuntimeError):
@@ -106,6 +106,12 @@ def _check(st, what):
 
 
 @dataclasses.dataclass
+class DPPoint(C.Structure):
+    _fields_ = [("makespan_s", C.c_double), ("energy_j", C.c_double), ("x64", C.c_double),
+                ("y64", C.c_double), ("score64", C.c_double), ("n_groups", C.c_int32),
+                ("group_of", C.c_int8 * 32), ("level_of", C.c_int8 * 32), ("valid", C.c_int32)]
+
+
 class SearchResult:
     status: int
     best: list            # [W] Pick (valid=0 if none)
@@ -212,6 +218,29 @@ class Scheduler:
         npv = min(npar.value, pareto_cap) if q.want_pareto else 0
         return SearchResult(rc, [best[w] for w in range(nw)], [par[k] for k in range(npv)],
                             stats.as_dict())
+
+    def front_dp(self, q, workspace=None, stream=None, front_cap=4096):
+        """Exact Pareto front and per-weight optimum of the whole space by the
+        device subset DP (sched_front_dp).  Returns (status, best[W], front,
+        stats); points carry one witness configuration (group_of, level_of)."""
+        import torch
+        n = C.c_size_t()
+        cq = self.cquery(q)
+        _check(lib().sched_dp_workspace_size(self._h, C.byref(cq), C.byref(n)), "sched_dp_workspace_size")
+        ws = workspace if workspace is not None else torch.empty(n.value, dtype=torch.uint8, device="cuda")
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        nw = len(q.weights)
+        best = (DPPoint * max(1, nw))()
+        front = (DPPoint * front_cap)()
+        nf = C.c_uint64()
+        stats = Stats()
+        rc = lib().sched_front_dp(self._h, C.byref(cq), C.c_void_p(ws.data_ptr()), C.c_size_t(ws.numel()),
+                                  C.c_void_p(st), best, front, C.c_uint64(front_cap), C.byref(nf),
+                                  C.byref(stats))
+        if rc not in (SCHED_OK, SCHED_E_INFEASIBLE):
+            raise SchedError(rc, "sched_front_dp")
+        return rc, [best[w] for w in range(nw)], [front[i] for i in range(min(nf.value, front_cap))], \
+            stats.as_dict()
 
     def heuristic(self, q, priority="throughput", w=0):
         """The paper's rule-based scheduler (criteria 1-4).
