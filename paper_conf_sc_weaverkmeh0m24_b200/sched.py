@@ -94,8 +94,9 @@ def lib():
             getattr(L, name)
         L.sched_strerror.restype = C.c_char_p
         L.sched_version.restype = C.c_char_p
-        for name in EXPORTS[:-2]:
-            getattr(L, name).restype = C.c_int
+        for name in EXPORTS:
+            if name not in ("sched_strerror", "sched_version"):
+                getattr(L, name).restype = C.c_int
         _lib = L
     return _lib
 
