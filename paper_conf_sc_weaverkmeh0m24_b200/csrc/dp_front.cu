@@ -140,6 +140,138 @@ __device__ __forceinline__ void decode_vec(const DevParams &p, uint32_t B, uint3
     }
 }
 
+// Split evaluation of a PER_CLIENT group's level vectors (L <= 4, |B| > kH):
+// the vector's digits split into the members' high part (all but the last kH
+// members, the most significant digits) and the low part (the last kH
+// members, highest workflow indices).  Every canonical sum runs over members
+// in ascending order, so the low members' terms come LAST: per high
+// assignment the high prefixes (U, B, D, each high member's sigma over the
+// other high members, each low member's sigma prefix over the high members
+// for each of its levels) are summed once, and each of the L^kH low vectors
+// only appends its terms -- the same additions in the same order as the
+// from-scratch evaluation (group64), hence the same fp64 bits.  T uses
+// max_i fl(fl(t_i s_i) c) = fl(c * max_i fl(t_i s_i)) (rounding is monotone).
+constexpr int kMS = 16;  // largest group on the split path
+constexpr int kH = 3;    // low members
+
+__device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, uint32_t B, int s, uint64_t v0,
+                                         uint64_t v1, int lane, PPt *f, int &nf, bool &ok) {
+  const int L = p.L, nh = s - kH;
+  const uint32_t Lh = (uint32_t)(L * L * L);
+  int mw[kMS];
+  {
+    int k = 0;
+#pragma unroll
+    for (int b = 0; b < 32; b++)
+      if (B >> b & 1u) {
+        if (k < kMS) mw[k] = b;
+        k++;
+      }
+  }
+  const double ps = p.ps;
+  for (uint64_t hv = v0 / Lh + lane; hv * Lh < v1; hv += 32) {
+    int rh[kMS - kH];
+    double sg[kMS - kH];
+    double U = 0.0, Bw = 0.0, D = 0.0;
+    {
+      uint64_t x = hv;
+#pragma unroll
+      for (int k = kMS - kH - 1; k >= 0; k--)
+        if (k < nh) {
+          rh[k] = mw[k] * L + (int)(x % (uint64_t)L);
+          x /= (uint64_t)L;
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < kMS - kH; k++)
+      if (k < nh) {
+        const int r = rh[k];
+        U = __dadd_rn(U, (double)tb.u[r]);
+        Bw = __dadd_rn(Bw, (double)tb.bw[r]);
+        D = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]));
+      }
+#pragma unroll
+    for (int k = 0; k < kMS - kH; k++)
+      if (k < nh) {
+        double a = 1.0;
+#pragma unroll
+        for (int q = 0; q < kMS - kH; q++)
+          if (q < nh && q != k) a = __dadd_rn(a, (double)tb.d[rh[k] * p.ds + rh[q]]);
+        sg[k] = a;
+      }
+    double Q[kH][4];  // low member j at level l: 1 + sum over the high members
+#pragma unroll
+    for (int j = 0; j < kH; j++)
+#pragma unroll
+      for (int l = 0; l < 4; l++) {
+        double a = 1.0;
+        if (l < L) {
+          const int rj = mw[nh + j] * L + l;
+#pragma unroll
+          for (int q = 0; q < kMS - kH; q++)
+            if (q < nh) a = __dadd_rn(a, (double)tb.d[rj * p.ds + rh[q]]);
+        }
+        Q[j][l] = a;
+      }
+    const uint64_t base = hv * Lh;
+    const uint32_t lv0 = (uint32_t)(v0 > base ? v0 - base : 0), lv1 = (uint32_t)(v1 - base < Lh ? v1 - base : Lh);
+    for (uint32_t lv = lv0; lv < lv1; lv++) {
+      int dl[kH], rl[kH];
+      {
+        uint32_t x = lv;
+#pragma unroll
+        for (int j = kH - 1; j >= 0; j--) {
+          dl[j] = (int)(x % (uint32_t)L);
+          x /= (uint32_t)L;
+          rl[j] = mw[nh + j] * L + dl[j];
+        }
+      }
+      double Ul = U, Bl = Bw, Dl = D;
+#pragma unroll
+      for (int j = 0; j < kH; j++) {
+        Ul = __dadd_rn(Ul, (double)tb.u[rl[j]]);
+        Bl = __dadd_rn(Bl, (double)tb.bw[rl[j]]);
+        Dl = __dadd_rn(Dl, __dmul_rn(__dsub_rn((double)tb.praw[rl[j]], ps), (double)tb.traw[rl[j]]));
+      }
+      if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Ul > 1.0 || Bl > 1.0)) continue;
+      double c = 1.0;
+      if (Ul > c) c = Ul;
+      if (Bl > c) c = Bl;
+      double mx = 0.0;
+#pragma unroll
+      for (int k = 0; k < kMS - kH; k++)
+        if (k < nh) {
+          double a = sg[k];
+          const int rd = rh[k] * p.ds;
+#pragma unroll
+          for (int j = 0; j < kH; j++) a = __dadd_rn(a, (double)tb.d[rd + rl[j]]);
+          const double ts = __dmul_rn((double)tb.traw[rh[k]], a);
+          if (ts > mx) mx = ts;
+        }
+#pragma unroll
+      for (int j = 0; j < kH; j++) {
+        double a = Q[j][dl[j]];
+#pragma unroll
+        for (int j2 = 0; j2 < kH; j2++)
+          if (j2 != j) a = __dadd_rn(a, (double)tb.d[rl[j] * p.ds + rl[j2]]);
+        const double ts = __dmul_rn((double)tb.traw[rl[j]], a);
+        if (ts > mx) mx = ts;
+      }
+      double Tg = __dmul_rn(mx, c);
+      if (p.model & SCHED_MODEL_POWER_CAP) {
+        const double tcap = __ddiv_rn(Dl, p.capd);
+        if (tcap > Tg) Tg = tcap;
+      }
+      PPt x;
+      x.t = Tg;
+      x.e = __dadd_rn(__dmul_rn(ps, Tg), Dl);
+      x.v = (uint32_t)(base + lv);
+      x.pad = 0;
+      ok &= front_insert<kLF>(f, nf, x);
+    }
+  }
+}
+
 // phase 1a: work item = (group, 2^kItemLog2 level vectors); one warp per item
 __global__ void __launch_bounds__(256) k_pf_items(const DpParams dp) {
   extern __shared__ __align__(16) unsigned char sm[];
@@ -168,13 +300,17 @@ __global__ void __launch_bounds__(256) k_pf_items(const DpParams dp) {
     int nf = 0;
     bool ok = true;
     int lev[kMaxN];
-    for (uint64_t v = v0 + lane; v < v1; v += 32) {
-      decode_vec(dp.p, B, (uint32_t)v, lev);
-      PPt x;
-      if (!group64(tb, dp.p, B, lev, x.t, x.e)) continue;
-      x.v = (uint32_t)v;
-      x.pad = 0;
-      ok &= front_insert<kLF>(f, nf, x);
+    if (dp.p.scope == SCHED_PER_CLIENT && s > kH && s <= kMS && dp.p.L <= 4) {
+      pf_split(tb, dp.p, B, s, v0, v1, lane, f, nf, ok);
+    } else {
+      for (uint64_t v = v0 + lane; v < v1; v += 32) {
+        decode_vec(dp.p, B, (uint32_t)v, lev);
+        PPt x;
+        if (!group64(tb, dp.p, B, lev, x.t, x.e)) continue;
+        x.v = (uint32_t)v;
+        x.pad = 0;
+        ok &= front_insert<kLF>(f, nf, x);
+      }
     }
     if (!ok) atomicExch(dp.ctr + kDpErr, 1ull);
     // warp merge: every lane keeps its points not dominated by another lane's
