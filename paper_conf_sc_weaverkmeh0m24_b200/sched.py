@@ -106,13 +106,13 @@ def _check(st, what):
         raise SchedError(st, what)
 
 
-@dataclasses.dataclass
 class DPPoint(C.Structure):
     _fields_ = [("makespan_s", C.c_double), ("energy_j", C.c_double), ("x64", C.c_double),
                 ("y64", C.c_double), ("score64", C.c_double), ("n_groups", C.c_int32),
                 ("group_of", C.c_int8 * 32), ("level_of", C.c_int8 * 32), ("valid", C.c_int32)]
 
 
+@dataclasses.dataclass
 class SearchResult:
     status: int
     best: list            # [W] Pick (valid=0 if none)

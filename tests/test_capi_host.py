@@ -209,3 +209,12 @@ def test_heuristic_rules_and_gap(seed):
         ok, T, E = oracle.score(prof, q, oa, od)
         assert pick.valid == ok and pick.makespan_s == T and pick.energy_j == E
         assert pick.score64 <= ref["best"][0][1]
+
+
+def test_binding_result_types_construct():
+    """The binding's result containers build from plain values (the ctypes
+    records stay plain Structures; SearchResult is a dataclass)."""
+    r = S.sched.SearchResult(0, [], [], {"n_configs": 0})
+    assert r.status == 0 and r.best_indices == [] and r.pareto_indices == []
+    p = S.sched.DPPoint()
+    assert p.valid == 0 and len(p.group_of) == 32
