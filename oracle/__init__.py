@@ -10,7 +10,9 @@ imports the other; both consume the seeded inputs of synth/.
              pure-Python fp64 score (N <= 6)
   enum.c     O1: recursive fp64 enumerator, index windows        [pinned]
              (ctypes wrapper below; parallel windows + merge)
-  dpcert.py  O3: exact subset-DP certificate of optimal values
+  dpcert.c   O3/O4: exact subset-DP certificate of optimal values
+  split.py   O5: scheduling-configuration (task split) search over the
+             split vectors of the queue (R29)
 """
 from __future__ import annotations
 
@@ -54,7 +56,8 @@ class _Query(C.Structure):
                 ("lev", C.POINTER(C.c_int)), ("scope", C.c_int), ("nw", C.c_int),
                 ("wa", C.POINTER(C.c_int)), ("wb", C.POINTER(C.c_int)),
                 ("lo", C.c_uint64), ("hi", C.c_uint64), ("want_pareto", C.c_int),
-                ("model", C.c_uint), ("power_cap", C.c_float)]
+                ("model", C.c_uint), ("power_cap", C.c_float),
+                ("tseq_base", C.c_double), ("eseq_base", C.c_double)]
 
 
 class _Best(C.Structure):
@@ -111,7 +114,8 @@ class _Pack:
         self.Q = _Query(q.n, q.g, min(q.c, q.n), len(q.levels), _ptr(lev, C.c_int),
                         q.scope, len(q.weights), _ptr(wa, C.c_int), _ptr(wb, C.c_int),
                         int(q.index_lo), int(hi), int(bool(q.want_pareto)),
-                        int(getattr(q, "model", 0)), float(getattr(q, "power_cap", 0.0)))
+                        int(getattr(q, "model", 0)), float(getattr(q, "power_cap", 0.0)),
+                        float(getattr(q, "tseq_base", 0.0)), float(getattr(q, "eseq_base", 0.0)))
 
 
 def count(q) -> int:

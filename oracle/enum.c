@@ -81,6 +81,8 @@ typedef struct {
   int want_pareto;
   unsigned model;          /* variant bits: 1 COUNT_IDLE, 2 NO_INTERFERENCE, 4 POWER_CAP */
   float power_cap;         /* P_cap (W) for POWER_CAP */
+  double tseq_base, eseq_base;  /* > 0: sequential baselines given by the caller (the unsplit
+                                   queue of a split search, R29); 0: computed below */
 } or_query;
 
 #define OR_COUNT_IDLE 1u
@@ -197,6 +199,8 @@ void oracle_constants(const or_profile *P, const or_query *q, int l100,
       E = E + e;
     }
   }
+  if (q->tseq_base > 0.0) T = q->tseq_base;   /* R29: baselines of the unsplit queue */
+  if (q->eseq_base > 0.0) E = q->eseq_base;
   *tseq = T; *eseq = E;
 }
 

@@ -24,6 +24,8 @@ class Query:
     index_hi: int | None = None   # None = |Omega|
     model: int = 0                # scoring-model variant bits (R26-R28): 1 COUNT_IDLE,
     power_cap: float = 0.0        # 2 NO_INTERFERENCE, 4 POWER_CAP (P_cap in W)
+    tseq_base: float = 0.0        # > 0: sequential baselines supplied by the caller (the
+    eseq_base: float = 0.0        # unsplit queue of a split search, R29)
 
     def with_range(self, lo, hi):
         return dataclasses.replace(self, index_lo=lo, index_hi=hi)
