@@ -249,6 +249,45 @@ int sched_front_dp(sched_handle *h, const sched_query *q, void *d_workspace, siz
 int sched_heuristic(const sched_handle *h, const sched_query *q, int32_t priority, int32_t w,
                     int8_t *group_of, int8_t *level_of, uint64_t *index, sched_pick *out);
 
+/* Scheduling-configuration search ("scheduling
+ * configuration ... the number of sequential tasks in each workflow as well as
+ * the number of concurrent workflows", L176 "split them into multiple parallel
+ * workflows", Figs 4-5 "s-p" labels; reading R29 in DESIGN.md).
+ * Workflow i of the query consists of tasks[i] >= 1 identical independent
+ * tasks (its profile row is the whole workflow).  A split vector p runs it as
+ * p_i concurrent MPS clients (p_i a divisor of tasks[i], p_i <= max_split[i]
+ * if max_split != NULL) of tasks[i]/p_i tasks each.  Split vectors are ranked
+ * lexicographically (divisors ascending, workflow 0 most significant).  For
+ * every split the expanded queue (clients workflow-major; client time
+ * fl32((t_i * s_i) / tasks[i]) at every level, the workflow's power, SM, BW
+ * and memory; co-run slowdown between siblings = the profile's diagonal
+ * block d[i,l][i,m]) is searched exhaustively on the device exactly as
+ * sched_search does, against the SAME sequential baselines T_seq, E_seq of
+ * the unsplit queue (q as given), so X and Y compare across splits.
+ * best[W]: max F per weight over all splits (ties -> lowest split rank, then
+ * lowest index in that split's space); pareto: the distinct (T, E) not
+ * dominated by any configuration of any split, one witness each (lowest
+ * (rank, index)), T ascending; *n_pareto as in sched_search (CAPACITY ->
+ * required size).  The query must cover the whole space of one shard
+ * (index window default, shard_count 1).  Every split must have <= 32
+ * clients and |Omega| <= 2^63 (else SCHED_E_TOO_LARGE: bound max_split).
+ * stats (may be NULL): sums over the splits; t_seq_s/e_seq_j = the unsplit
+ * baselines.  Workspace: sched_split_workspace_size (the max over splits),
+ * which also returns the number of split vectors. */
+typedef struct {
+  sched_pick pick;                     /* index in the expanded space of split `split_rank` */
+  uint32_t split_rank;                 /* rank of the split vector */
+  int32_t n_clients;                   /* sum of split[0..n) */
+  int32_t split[SCHED_MAX_WORKFLOWS];  /* p_i: concurrent clients of workflow i */
+} sched_split_pick;
+
+int sched_split_workspace_size(const sched_handle *h, const sched_query *q, const int32_t *tasks,
+                               const int32_t *max_split, size_t *bytes, uint32_t *n_splits);
+int sched_search_splits(sched_handle *h, const sched_query *q, const int32_t *tasks,
+                        const int32_t *max_split, void *d_workspace, size_t ws_bytes, void *cuda_stream,
+                        sched_split_pick *best, sched_split_pick *pareto, uint64_t pareto_cap,
+                        uint64_t *n_pareto, sched_stats *stats);
+
 const char *sched_strerror(int status);
 
 /* Library version string, e.g. "sched-b200 0.1 sm_100a". */

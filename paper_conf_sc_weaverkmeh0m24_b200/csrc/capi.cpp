@@ -117,6 +117,22 @@ void fill_pick(const Query &q, const DevParams &dp, int w, const BestRec &b, sch
   o->score32 = s;
 }
 
+// split search setup (R29): admissible split vectors and the unsplit baselines
+int split_setup(sched_handle *h, const sched_query *qin, const int32_t *tasks, const int32_t *max_split,
+                std::vector<std::vector<int>> *svs, double *tseq, double *eseq) {
+  if (!h || !qin || !tasks) return SCHED_E_INVALID;
+  Query q;
+  int st = resolve_query_shape(qin, h->P.lp, &q);
+  if (st) return st;
+  if (q.n > h->P.n) return SCHED_E_INVALID;
+  if ((q.model & SCHED_MODEL_POWER_CAP) && !(q.pcap > h->P.ps)) return SCHED_E_INVALID;
+  if (qin->index_lo != 0 || qin->index_hi != UINT64_MAX || q.count != 1) return SCHED_E_INVALID;
+  st = split_vectors(q.n, tasks, max_split, svs);
+  if (st) return st;
+  host_constants(h->P, q, tseq, eseq);
+  return SCHED_OK;
+}
+
 }  // namespace
 
 #define GUARD_BEGIN try {
@@ -517,6 +533,148 @@ int sched_heuristic(const sched_handle *hc, const sched_query *qin, int32_t prio
   out->y64 = es / E;
   const int ea = q.nw ? q.wa[w] : 1, eb = q.nw ? q.wb[w] : 0;
   out->score64 = host_objective(ts, es, T, E, ea, eb);
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_split_workspace_size(const sched_handle *hc, const sched_query *qin, const int32_t *tasks,
+                               const int32_t *max_split, size_t *bytes, uint32_t *n_splits) {
+  GUARD_BEGIN
+  if (!bytes) return SCHED_E_INVALID;
+  sched_handle *h = const_cast<sched_handle *>(hc);
+  std::vector<std::vector<int>> svs;
+  double tseq, eseq;
+  int st = split_setup(h, qin, tasks, max_split, &svs, &tseq, &eseq);
+  if (st) return st;
+  size_t mx = 0;
+  sched_handle tmp;
+  for (const auto &sv : svs) {
+    st = expand_split(h->P, qin->n, tasks, sv, &tmp.P);
+    if (st) return st;
+    tmp.sp_key[0] = -1;
+    sched_query q2 = *qin;
+    q2.n = tmp.P.n;
+    size_t b = 0;
+    st = sched_workspace_size(&tmp, &q2, &b);
+    if (st) return st;
+    mx = std::max(mx, b);
+  }
+  *bytes = mx;
+  if (n_splits) *n_splits = (uint32_t)svs.size();
+  return SCHED_OK;
+  GUARD_END
+}
+
+int sched_search_splits(sched_handle *h, const sched_query *qin, const int32_t *tasks, const int32_t *max_split,
+                        void *ws, size_t ws_bytes, void *stream, sched_split_pick *best,
+                        sched_split_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto,
+                        sched_stats *stats) {
+  GUARD_BEGIN
+  if (!ws) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  std::vector<std::vector<int>> svs;
+  double tseq, eseq;
+  st = split_setup(h, qin, tasks, max_split, &svs, &tseq, &eseq);
+  if (st) return st;
+  const int nw = qin->n_weights, n = qin->n;
+  const bool want_par = qin->want_pareto != 0;
+  if (nw > 0 && !best) return SCHED_E_INVALID;
+  if (want_par && (!n_pareto || (pareto_cap > 0 && !pareto))) return SCHED_E_INVALID;
+  auto fill_split = [&](sched_split_pick *o, const sched_pick &pk, uint32_t r) {
+    std::memset(o, 0, sizeof *o);
+    o->pick = pk;
+    o->split_rank = r;
+    for (int i = 0; i < n; i++) o->n_clients += (o->split[i] = svs[r][i]);
+  };
+  std::vector<sched_split_pick> bst(std::max(nw, 1));
+  for (auto &b : bst) std::memset(&b, 0, sizeof b);
+  struct PP {
+    double t, e;
+    uint32_t r;
+    uint64_t idx;
+    sched_pick pk;
+  };
+  std::vector<PP> pts;
+  sched_stats agg;
+  std::memset(&agg, 0, sizeof agg);
+  sched_handle tmp;
+  std::vector<sched_pick> pb(std::max(nw, 1)), pp(4096);
+  int rc = SCHED_OK;
+  for (uint32_t r = 0; r < svs.size() && rc == SCHED_OK; r++) {
+    st = expand_split(h->P, n, tasks, svs[r], &tmp.P);
+    if (st) { rc = st; break; }
+    tmp.P.tseq_base = tseq;
+    tmp.P.eseq_base = eseq;
+    tmp.sp_key[0] = -1;
+    tmp.staged_ws = nullptr;
+    sched_query q2 = *qin;
+    q2.n = tmp.P.n;
+    uint64_t np = 0;
+    sched_stats s1;
+    for (;;) {
+      st = sched_search(&tmp, &q2, ws, ws_bytes, stream, pb.data(), pp.data(), pp.size(), &np, &s1);
+      if (st == SCHED_E_CAPACITY && want_par && np > pp.size()) {
+        pp.resize(np);
+        continue;
+      }
+      break;
+    }
+    if (st && st != SCHED_E_INFEASIBLE) { rc = st; break; }
+    agg.n_configs += s1.n_configs;
+    agg.n_feasible += s1.n_feasible;
+    agg.n_refined += s1.n_refined;
+    agg.n_candidates += s1.n_candidates;
+    agg.search_ms += s1.search_ms;
+    agg.total_ms += s1.total_ms;
+    agg.kernel_launches += s1.kernel_launches;
+    agg.passes += s1.passes;
+    agg.h2d_bytes += s1.h2d_bytes;
+    agg.d2h_bytes += s1.d2h_bytes;
+    agg.grid_ctas = std::max(agg.grid_ctas, s1.grid_ctas);
+    agg.kernel_path = s1.kernel_path;
+    if (st == SCHED_E_INFEASIBLE) continue;
+    for (int w = 0; w < nw; w++) {
+      const sched_pick &c = pb[w];
+      if (!c.valid) continue;
+      // ranks ascend: a later split replaces only on a strictly greater score
+      if (!bst[w].pick.valid || c.score64 > bst[w].pick.score64) fill_split(&bst[w], c, r);
+    }
+    if (want_par)
+      for (uint64_t k = 0; k < np; k++) pts.push_back({pp[k].makespan_s, pp[k].energy_j, r, pp[k].index, pp[k]});
+  }
+  if (tmp.pinned) cudaFreeHost(tmp.pinned);
+  tmp.pinned = nullptr;
+  if (rc) return rc;
+  for (int w = 0; w < nw; w++) best[w] = bst[w];
+  uint64_t nf = 0;
+  if (want_par) {
+    std::sort(pts.begin(), pts.end(), [](const PP &a, const PP &b) {
+      if (a.t != b.t) return a.t < b.t;
+      if (a.e != b.e) return a.e < b.e;
+      if (a.r != b.r) return a.r < b.r;
+      return a.idx < b.idx;
+    });
+    bool have = false;
+    double bestE = 0.0;
+    for (const PP &x : pts) {
+      if (have && !(x.e < bestE)) continue;
+      have = true;
+      bestE = x.e;
+      if (nf < pareto_cap) fill_split(&pareto[nf], x.pk, x.r);
+      nf++;
+    }
+    *n_pareto = nf;
+  } else if (n_pareto) {
+    *n_pareto = 0;
+  }
+  if (stats) {
+    *stats = agg;
+    stats->t_seq_s = tseq;
+    stats->e_seq_j = eseq;
+  }
+  if (want_par && nf > pareto_cap) return SCHED_E_CAPACITY;
+  if (agg.n_feasible == 0) return SCHED_E_INFEASIBLE;
   return SCHED_OK;
   GUARD_END
 }

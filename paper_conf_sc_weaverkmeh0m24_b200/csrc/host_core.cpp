@@ -351,8 +351,85 @@ void host_constants(const Profile &P, const Query &q, double *tseq, double *eseq
       E = E + e;
     }
   }
+  if (P.tseq_base > 0.0) T = P.tseq_base;  // R29: the unsplit queue's baselines
+  if (P.eseq_base > 0.0) E = P.eseq_base;
   *tseq = T;
   *eseq = E;
+}
+
+// ------------------------------------------------------------ task splits (R29)
+// Workflow i = tasks[i] identical independent tasks (Table III "# Iter.",
+// R17); a split runs it as p_i | tasks[i] concurrent clients of
+// tasks[i]/p_i tasks each ("split them into multiple
+// parallel workflows"; Figs 4-5 "s-p").  Split vectors are ranked
+// lexicographically, divisors ascending, workflow 0 most significant.
+int split_vectors(int n, const int32_t *tasks, const int32_t *max_split, std::vector<std::vector<int>> *out) {
+  if (!tasks || n < 1 || n > kMaxN) return SCHED_E_INVALID;
+  std::vector<std::vector<int>> ch(n);
+  uint64_t total = 1;
+  for (int i = 0; i < n; i++) {
+    if (tasks[i] < 1 || tasks[i] > (1 << 20)) return SCHED_E_INVALID;
+    const int lim = max_split ? max_split[i] : tasks[i];
+    if (lim < 1) return SCHED_E_INVALID;
+    for (int d = 1; d <= tasks[i] && d <= lim && d <= kMaxN; d++)
+      if (tasks[i] % d == 0) ch[i].push_back(d);
+    total *= ch[i].size();
+    if (total > (1u << 20)) return SCHED_E_TOO_LARGE;
+  }
+  out->clear();
+  std::vector<int> pos(n, 0);
+  for (;;) {  // odometer, last workflow fastest
+    std::vector<int> v(n);
+    int sum = 0;
+    for (int i = 0; i < n; i++) sum += (v[i] = ch[i][pos[i]]);
+    if (sum > kMaxN) return SCHED_E_TOO_LARGE;  // more clients than a query takes: cap with max_split
+    out->push_back(v);
+    int i = n - 1;
+    while (i >= 0 && ++pos[i] == (int)ch[i].size()) pos[i--] = 0;
+    if (i < 0) break;
+  }
+  return SCHED_OK;
+}
+
+// Expanded client queue (workflow-major): client of workflow i runs
+// fl32((t_i * s_i) / K_i) at every level, same power / SM / BW / memory;
+// co-run d between clients of workflows i, j is d[i,l][j,m] (siblings: the
+// profile's diagonal block, the self co-run slowdown).
+int expand_split(const Profile &P, int n, const int32_t *tasks, const std::vector<int> &split, Profile *E) {
+  std::vector<int> own;
+  for (int i = 0; i < n; i++)
+    for (int r = 0; r < split[i]; r++) own.push_back(i);
+  const int m = (int)own.size(), lp = P.lp;
+  if (m < 1 || m > kMaxN) return SCHED_E_TOO_LARGE;
+  E->n = m;
+  E->lp = lp;
+  E->pct = P.pct;
+  E->l100 = P.l100;
+  E->mem_cap = P.mem_cap;
+  E->ps = P.ps;
+  E->tseq_base = E->eseq_base = 0.0;
+  E->t.resize((size_t)m * lp);
+  E->p.resize((size_t)m * lp);
+  E->u.resize((size_t)m * lp);
+  E->bw.resize((size_t)m * lp);
+  E->mem.resize(m);
+  E->d.resize((size_t)m * lp * m * lp);
+  for (int a = 0; a < m; a++) {
+    const int i = own[a];
+    const double K = (double)tasks[i], s = (double)(tasks[i] / split[i]);
+    for (int l = 0; l < lp; l++) {
+      const size_t src = (size_t)i * lp + l, dst = (size_t)a * lp + l;
+      E->t[dst] = (float)(((double)P.t[src] * s) / K);
+      E->p[dst] = P.p[src];
+      E->u[dst] = P.u[src];
+      E->bw[dst] = P.bw[src];
+      for (int b = 0; b < m; b++)
+        for (int mm = 0; mm < lp; mm++)
+          E->d[(dst * m + b) * lp + mm] = P.d[(src * P.n + own[b]) * lp + mm];
+    }
+    E->mem[a] = P.mem[i];
+  }
+  return SCHED_OK;
 }
 
 // Canonical score (PAPER.md L87 predicate + memory clause, L91, L96).

@@ -33,6 +33,9 @@ struct Profile {
   int mem_cap = 0;
   float ps = 0.f;
   int l100 = -1;
+  // > 0: sequential baselines fixed by the caller instead of computed from
+  // this profile (the unsplit queue of a split search, R29)
+  double tseq_base = 0.0, eseq_base = 0.0;
 };
 
 // Validated query (levels resolved to profile level indices).
@@ -159,6 +162,10 @@ void host_constants(const Profile &P, const Query &q, double *tseq, double *eseq
 int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const int8_t *digits,
                double *T, double *E);
 double host_objective(double tseq, double eseq, double T, double E, int a, int b);
+// scheduling-configuration split (R29): admissible
+// split vectors in rank order, and the expanded client profile of one
+int split_vectors(int n, const int32_t *tasks, const int32_t *max_split, std::vector<std::vector<int>> *out);
+int expand_split(const Profile &P, int n, const int32_t *tasks, const std::vector<int> &split, Profile *out);
 // staged table blob + DevParams (work split, bounds) for one query
 int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<unsigned char> *blob,
                 DevParams *dp);

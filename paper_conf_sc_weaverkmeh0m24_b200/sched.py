@@ -32,7 +32,8 @@ UINT64_MAX = (1 << 64) - 1
 
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
            "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score", "sched_heuristic",
-           "sched_strerror", "sched_version", "sched_dp_workspace_size", "sched_front_dp"]
+           "sched_strerror", "sched_version", "sched_dp_workspace_size", "sched_front_dp",
+           "sched_split_workspace_size", "sched_search_splits"]
 
 
 class SchedError(RuntimeError):
@@ -110,6 +111,11 @@ class DPPoint(C.Structure):
     _fields_ = [("makespan_s", C.c_double), ("energy_j", C.c_double), ("x64", C.c_double),
                 ("y64", C.c_double), ("score64", C.c_double), ("n_groups", C.c_int32),
                 ("group_of", C.c_int8 * 32), ("level_of", C.c_int8 * 32), ("valid", C.c_int32)]
+
+
+class SplitPick(C.Structure):
+    _fields_ = [("pick", Pick), ("split_rank", C.c_uint32), ("n_clients", C.c_int32),
+                ("split", C.c_int32 * 32)]
 
 
 @dataclasses.dataclass
@@ -242,6 +248,39 @@ class Scheduler:
             raise SchedError(rc, "sched_front_dp")
         return rc, [best[w] for w in range(nw)], [front[i] for i in range(min(nf.value, front_cap))], \
             stats.as_dict()
+
+    def search_splits(self, q, tasks, max_split=None, stream=None, pareto_cap=4096):
+        """Scheduling-configuration search (sched_search_splits; SURVEY 8(f) N3,
+        DESIGN.md R29): every split of workflow i's tasks[i] tasks into
+        concurrent clients x every configuration of the expanded queue.
+        Returns (status, best[W], pareto, stats, n_splits); picks are
+        SplitPick (pick, split_rank, n_clients, split[])."""
+        import torch
+        t = _i32(tasks)
+        ms = None if max_split is None else _i32(max_split)
+        tp = t.ctypes.data_as(C.POINTER(C.c_int32))
+        mp = None if ms is None else ms.ctypes.data_as(C.POINTER(C.c_int32))
+        cq = self.cquery(q)
+        n = C.c_size_t()
+        ns = C.c_uint32()
+        _check(lib().sched_split_workspace_size(self._h, C.byref(cq), tp, mp, C.byref(n), C.byref(ns)),
+               "sched_split_workspace_size")
+        if self._ws is None or self._ws.numel() < n.value:
+            self._ws = torch.empty(n.value, dtype=torch.uint8, device="cuda")
+        ws = self._ws
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        nw = len(q.weights)
+        best = (SplitPick * max(1, nw))()
+        par = (SplitPick * max(1, pareto_cap))()
+        npar = C.c_uint64()
+        stats = Stats()
+        rc = lib().sched_search_splits(self._h, C.byref(cq), tp, mp, C.c_void_p(ws.data_ptr()),
+                                       C.c_size_t(ws.numel()), C.c_void_p(st), best, par,
+                                       C.c_uint64(pareto_cap), C.byref(npar), C.byref(stats))
+        if rc not in (SCHED_OK, SCHED_E_INFEASIBLE):
+            raise SchedError(rc, "sched_search_splits")
+        npv = min(npar.value, pareto_cap) if q.want_pareto else 0
+        return rc, [best[w] for w in range(nw)], [par[k] for k in range(npv)], stats.as_dict(), ns.value
 
     def heuristic(self, q, priority="throughput", w=0):
         """The paper's rule-based scheduler (criteria 1-4).

@@ -218,3 +218,35 @@ def test_binding_result_types_construct():
     assert r.status == 0 and r.best_indices == [] and r.pareto_indices == []
     p = S.sched.DPPoint()
     assert p.valid == 0 and len(p.group_of) == 32
+
+
+def test_split_pick_layout():
+    """sched_split_pick: sched_pick + rank + count + 32 split entries."""
+    assert C.sizeof(S.sched.SplitPick) == C.sizeof(S.sched.Pick) + 8 + 4 * 32
+    r = S.sched.SplitPick()
+    assert r.pick.valid == 0 and r.n_clients == 0
+
+
+def test_split_workspace_and_errors_host():
+    """Host-side split setup: count of split vectors (divisor product),
+    TOO_LARGE when a split exceeds 32 clients, INVALID for a windowed query."""
+    prof = make_profile(3, levels=(50, 100), seed=2)
+    q = Query(3, 2, 8, (50, 100), PER_GPU, ((1, 1),))
+    sch = S.Scheduler(prof)
+    cq = sch.cquery(q)
+    n = C.c_size_t()
+    ns = C.c_uint32()
+    t = np.array([4, 6, 1], np.int32)
+    tp = t.ctypes.data_as(C.POINTER(C.c_int32))
+    assert S.lib().sched_split_workspace_size(sch._h, C.byref(cq), tp, None, C.byref(n), C.byref(ns)) == 0
+    assert ns.value == 3 * 4 * 1 and n.value > 0
+    big = np.array([32, 2, 1], np.int32)
+    assert S.lib().sched_split_workspace_size(sch._h, C.byref(cq), big.ctypes.data_as(C.POINTER(C.c_int32)),
+                                              None, C.byref(n), C.byref(ns)) == S.sched.SCHED_E_TOO_LARGE
+    cap = np.array([2, 2, 1], np.int32)
+    assert S.lib().sched_split_workspace_size(sch._h, C.byref(cq), big.ctypes.data_as(C.POINTER(C.c_int32)),
+                                              cap.ctypes.data_as(C.POINTER(C.c_int32)), C.byref(n),
+                                              C.byref(ns)) == 0 and ns.value == 4
+    cw = sch.cquery(q.with_range(0, 10))
+    assert S.lib().sched_split_workspace_size(sch._h, C.byref(cw), tp, None, C.byref(n),
+                                              C.byref(ns)) == S.sched.SCHED_E_INVALID
