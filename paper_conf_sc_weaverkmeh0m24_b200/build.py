@@ -20,7 +20,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off,-fno-fast-math",
-          "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", CSRC]
+          "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
+          *os.environ.get("SCHED_NVCC_EXTRA", "").split()]
 
 
 def sources():

@@ -368,7 +368,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
 }
 
 template <int L, class WS>
-__global__ void __launch_bounds__(kTileThreads, 2) k_tile(const DevParams p) {
+__global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const DevParams p) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, p);
   const Tables tb = tables_at(sm, p);

@@ -25,7 +25,14 @@ struct TileLaunch {
   size_t smem;
 };
 
-constexpr int kTileThreads = 256;
+#ifndef SCHED_TILE_THREADS
+#define SCHED_TILE_THREADS 256
+#endif
+#ifndef SCHED_TILE_MINB
+#define SCHED_TILE_MINB 2
+#endif
+constexpr int kTileThreads = SCHED_TILE_THREADS;
+constexpr int kTileMinBlocks = SCHED_TILE_MINB;  // __launch_bounds__ min blocks per SM
 constexpr int kTileWarps = kTileThreads / 32;
 constexpr int kTileMaxL = 4;
 constexpr int kTileMaxG = 8;

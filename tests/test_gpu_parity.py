@@ -251,3 +251,25 @@ def test_dense_local_front_window():
     assert [(b.index, b.score64) for b in mb] == [(b.index, b.score64) for b in res.best]
     assert [(p.index, p.makespan_s, p.energy_j) for p in mp] == \
         [(p.index, p.makespan_s, p.energy_j) for p in res.pareto]
+
+
+@pytest.mark.parametrize("n,g,c,levels,scope", [
+    (32, 2, 32, (100,), PER_GPU),          # maximum queue (SCHED_MAX_WORKFLOWS), 2^31 configurations
+    (32, 16, 2, (100,), PER_GPU),          # maximum GPUs, pairs only: 32!/(2^16 16!) = 1.9e17
+    (20, 16, 48, (50, 100), PER_GPU),      # maximum GPUs and MPS clients, no group table cap
+    (13, 3, 13, (10, 20, 30, 40, 55, 70, 85, 100), PER_CLIENT),  # 8 searched levels (SCHED_MAX_SEARCH_LEVELS)
+])
+def test_maximum_sizes_windows(n, g, c, levels, scope):
+    """Maximum sizes of the boundary (include/sched.h): windows at the start,
+    the end and a ragged interior offset, bitwise against the oracle."""
+    lv = tuple(sorted(set(levels)))
+    # small-memory archetypes (Table II 1x rows) keep the large queues feasible
+    arch = [(0, 3, 5, 9)[i % 4] for i in range(n)] if n >= 20 else None
+    prof = make_profile(n, levels=lv, seed=900 + n + g, archetypes=arch)
+    q = Query(n, g, c, lv, scope, ((1, 0), (1, 1), (0, 1)), True)
+    tot = S.count(q)
+    assert tot == oracle.count(q) and tot < 1 << 63
+    sch = S.Scheduler(prof)
+    for lo in (0, tot // 3 + 12345, tot - 150_000):
+        qw = q.with_range(lo, min(tot, lo + 150_000))
+        check(sch.search(qw), oracle.search(prof, qw), qw)
