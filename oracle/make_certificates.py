@@ -1,10 +1,13 @@
 """Write tests/golden/<cfg>_certificate.json from the O3 subset-DP certificate
 (calls only oracle/ and the seeded input generator; TEST INFRASTRUCTURE).
 
-  python -m oracle.make_certificates
+  python -m oracle.make_certificates            # c3, c4, c5 (O3)
+  python -m oracle.make_certificates client 14  # O4: the first 14 workflows of c4, per-client levels
 """
+import dataclasses
 import json
 import os
+import sys
 
 import oracle
 from synth import config
@@ -26,5 +29,27 @@ def main():
         print(name, len(c["front"]), c["best"])
 
 
+def client(n: int):
+    """O4 (PER_CLIENT) certificate of the c4 profile's first n workflows with
+    c4's G = 8, 4 levels, uncapped clients: the literal per-client reading
+    at the largest size O4 can run (n = 14: 5^14 level-vector groups)."""
+    prof, q = config("c4")
+    q = dataclasses.replace(q, n=n, scope=0, weights=((1, 1), (2, 1), (1, 0), (0, 1)))
+    c = oracle.dp_certificate(prof.subset(n), q)
+    out = {"config": f"c4 first {n} workflows, PER_CLIENT", "n": n, "g": q.g, "c": q.c,
+           "levels": list(q.levels), "scope": "PER_CLIENT",
+           "source": "oracle.dp_certificate (oracle/dpcert.c, O4), seed 0 synth.config('c4').subset(n)",
+           "weights": [list(w) for w in q.weights],
+           "tseq": c["tseq"].hex(), "eseq": c["eseq"].hex(),
+           "best_score64": [b.hex() for b in c["best"]],
+           "front_T_E": [[t.hex(), e.hex()] for t, e in c["front"]],
+           "front_decimal": [[t, e] for t, e in c["front"]]}
+    json.dump(out, open(os.path.join(GOLD, f"c4_client_n{n}_certificate.json"), "w"), indent=1)
+    print(n, len(c["front"]), c["best"])
+
+
 if __name__ == "__main__":
-    main()
+    if len(sys.argv) > 2 and sys.argv[1] == "client":
+        client(int(sys.argv[2]))
+    else:
+        main()

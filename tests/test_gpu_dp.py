@@ -84,3 +84,24 @@ def test_dp_front_c4_literal_per_client():
         assert best[w].score64 >= bg[w].score64
     print("c4 per-client:", st["search_ms"], "ms;", len(front), "front points;",
           [b.score64 for b in best], "vs per-GPU", [b.score64 for b in bg])
+
+
+@pytest.mark.parametrize("n", [13, 14])
+def test_dp_front_c4_client_prefix_golden(n):
+    """Literal per-client reading on the c4 profile at the largest sizes the
+    O4 oracle runs (the first 13 / 14 workflows, G = 8, 4 levels per client:
+    5.9e13 / 7.3e14+ configurations): front values and optimum per weight
+    bitwise equal to the stored certificate (tests/golden, written by
+    `python -m oracle.make_certificates client n`)."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"c4_client_n{n}_certificate.json")))
+    prof, q = config("c4")
+    q = dataclasses.replace(q, n=n, scope=PER_CLIENT, weights=tuple(tuple(w) for w in g["weights"]))
+    p = prof.subset(n)
+    rc, best, front, st = S.Scheduler(p).front_dp(q)
+    assert rc == S.sched.SCHED_OK and st["kernel_path"] == 4
+    assert [[x.makespan_s.hex(), x.energy_j.hex()] for x in front] == g["front_T_E"]
+    assert [b.score64.hex() for b in best] == g["best_score64"]
+    for x in list(front) + list(best):
+        assert _witness_ok(p, q, x)
