@@ -417,11 +417,11 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
-    u64 ver_pref = p.want_pareto ? __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0) : 0;
+    u64 ver_pref = p.want_pareto ? __ldcg(p.ctr + kCtrStairVer) : 0;  // stair_sync broadcasts lane 0's
     for (;;) {
       if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
         stair_sync(stair, p, stair_ver, ver_pref);
-        ver_pref = __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0);
+        ver_pref = __ldcg(p.ctr + kCtrStairVer);  // consumed next partition: load latency off the path
       }
       const u64 base = wp.base;
       const uint32_t Pn = (uint32_t)wp.cfg.Pn;
