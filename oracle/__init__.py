@@ -13,6 +13,12 @@ imports the other; both consume the seeded inputs of synth/.
   dpcert.c   O3/O4: exact subset-DP certificate of optimal values
   split.py   O5: scheduling-configuration (task split) search over the
              split vectors of the queue (R29)
+
+Every function above is pinned by tests that do not re-type it (closed forms,
+brute force, hand-derived configurations, the paper's Table II/III numbers).
+Parity unpinned: whether the model's predicted X, Y agree with the paper's
+MEASURED Figs 2-5 -- the paper prints neither a prediction model nor numbers
+for those figures.
 """
 from __future__ import annotations
 
