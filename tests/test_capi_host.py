@@ -250,3 +250,32 @@ def test_split_workspace_and_errors_host():
     cw = sch.cquery(q.with_range(0, 10))
     assert S.lib().sched_split_workspace_size(sch._h, C.byref(cw), tp, None, C.byref(n),
                                               C.byref(ns)) == S.sched.SCHED_E_INVALID
+
+
+@pytest.mark.skipif(__import__("torch").cuda.is_available(), reason="checks the no-device path")
+def test_no_device_no_fallback():
+    """Without a GPU every compute entry point returns SCHED_E_NODEVICE before
+    touching the workspace: there is no CPU fallback."""
+    prof, q = config("c1")
+    sch = S.Scheduler(prof)
+    cq = sch.cquery(q)
+    fake = C.c_void_p(0x1000)   # never dereferenced
+    best = (S.sched.Pick * 4)()
+    par = (S.sched.Pick * 16)()
+    npar = C.c_uint64()
+    rc = S.lib().sched_search(sch._h, C.byref(cq), fake, C.c_size_t(1 << 30), None, best, par,
+                              C.c_uint64(16), C.byref(npar), None)
+    assert rc == S.sched.SCHED_E_NODEVICE
+    dp = (S.sched.DPPoint * 4)()
+    fr = (S.sched.DPPoint * 16)()
+    rc = S.lib().sched_front_dp(sch._h, C.byref(cq), fake, C.c_size_t(1 << 30), None, dp, fr,
+                                C.c_uint64(16), C.byref(npar), None)
+    assert rc == S.sched.SCHED_E_NODEVICE
+    t = np.array([2, 2, 1, 1], np.int32)
+    sb = (S.sched.SplitPick * 4)()
+    sp = (S.sched.SplitPick * 16)()
+    rc = S.lib().sched_search_splits(sch._h, C.byref(cq), t.ctypes.data_as(C.POINTER(C.c_int32)), None,
+                                     fake, C.c_size_t(1 << 30), None, sb, sp, C.c_uint64(16),
+                                     C.byref(npar), None)
+    assert rc == S.sched.SCHED_E_NODEVICE
+    assert S.lib().sched_strerror(S.sched.SCHED_E_NODEVICE)
