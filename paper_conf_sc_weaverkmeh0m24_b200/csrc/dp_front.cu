@@ -215,6 +215,70 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
       }
     const uint64_t base = hv * Lh;
     const uint32_t lv0 = (uint32_t)(v0 > base ? v0 - base : 0), lv1 = (uint32_t)(v1 - base < Lh ? v1 - base : Lh);
+    if (lv0 == 0 && lv1 == Lh) {
+      // Whole low block, nested over the low members' digits (d0 most
+      // significant, as the index): every partial sum that does not involve
+      // a deeper low member is formed once at its loop level -- the same
+      // additions in the same ascending-member order as below.
+      const int r0b = mw[nh] * L, r1b = mw[nh + 1] * L, r2b = mw[nh + 2] * L;
+      for (int d0 = 0; d0 < L; d0++) {
+        const int r0 = r0b + d0;
+        const double U0 = __dadd_rn(U, (double)tb.u[r0]), B0 = __dadd_rn(Bw, (double)tb.bw[r0]);
+        const double D0 = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r0], ps), (double)tb.traw[r0]));
+        double a0[kMS - kH];
+#pragma unroll
+        for (int k = 0; k < kMS - kH; k++)
+          if (k < nh) a0[k] = __dadd_rn(sg[k], (double)tb.d[rh[k] * p.ds + r0]);
+        for (int d1 = 0; d1 < L; d1++) {
+          const int r1 = r1b + d1;
+          const double U1 = __dadd_rn(U0, (double)tb.u[r1]), B1 = __dadd_rn(B0, (double)tb.bw[r1]);
+          const double D1 = __dadd_rn(D0, __dmul_rn(__dsub_rn((double)tb.praw[r1], ps), (double)tb.traw[r1]));
+          double a1[kMS - kH];
+#pragma unroll
+          for (int k = 0; k < kMS - kH; k++)
+            if (k < nh) a1[k] = __dadd_rn(a0[k], (double)tb.d[rh[k] * p.ds + r1]);
+          const double s0p = __dadd_rn(Q[0][d0], (double)tb.d[r0 * p.ds + r1]);  // low 0: + low 1
+          const double s1p = __dadd_rn(Q[1][d1], (double)tb.d[r1 * p.ds + r0]);  // low 1: + low 0
+          for (int d2 = 0; d2 < L; d2++) {
+            const int r2 = r2b + d2;
+            const double Ul = __dadd_rn(U1, (double)tb.u[r2]), Bl = __dadd_rn(B1, (double)tb.bw[r2]);
+            const double Dl =
+                __dadd_rn(D1, __dmul_rn(__dsub_rn((double)tb.praw[r2], ps), (double)tb.traw[r2]));
+            if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Ul > 1.0 || Bl > 1.0)) continue;
+            double c = 1.0;
+            if (Ul > c) c = Ul;
+            if (Bl > c) c = Bl;
+            double mx = 0.0;
+#pragma unroll
+            for (int k = 0; k < kMS - kH; k++)
+              if (k < nh) {
+                const double ts =
+                    __dmul_rn((double)tb.traw[rh[k]], __dadd_rn(a1[k], (double)tb.d[rh[k] * p.ds + r2]));
+                if (ts > mx) mx = ts;
+              }
+            const double t0 = __dmul_rn((double)tb.traw[r0], __dadd_rn(s0p, (double)tb.d[r0 * p.ds + r2]));
+            const double t1 = __dmul_rn((double)tb.traw[r1], __dadd_rn(s1p, (double)tb.d[r1 * p.ds + r2]));
+            const double t2 = __dmul_rn((double)tb.traw[r2], __dadd_rn(__dadd_rn(Q[2][d2], (double)tb.d[r2 * p.ds + r0]),
+                                                                    (double)tb.d[r2 * p.ds + r1]));
+            if (t0 > mx) mx = t0;
+            if (t1 > mx) mx = t1;
+            if (t2 > mx) mx = t2;
+            double Tg = __dmul_rn(mx, c);
+            if (p.model & SCHED_MODEL_POWER_CAP) {
+              const double tcap = __ddiv_rn(Dl, p.capd);
+              if (tcap > Tg) Tg = tcap;
+            }
+            PPt x;
+            x.t = Tg;
+            x.e = __dadd_rn(__dmul_rn(ps, Tg), Dl);
+            x.v = (uint32_t)(base + (uint32_t)((d0 * L + d1) * L + d2));
+            x.pad = 0;
+            ok &= front_insert<kLF>(f, nf, x);
+          }
+        }
+      }
+      continue;
+    }
     for (uint32_t lv = lv0; lv < lv1; lv++) {
       int dl[kH], rl[kH];
       {
