@@ -33,6 +33,10 @@
 
 namespace sched {
 
+#ifndef SCHED_PF_MINB
+#define SCHED_PF_MINB 2  // k_pf_items CTAs per SM the register budget is sized for (1: 3.97 s, 2: 2.66 s)
+#endif
+
 constexpr int kLF = 16;     // lane-local front capacity (phase 1)
 constexpr int kOF = 16;     // per work item / per group front capacity
 constexpr int kFM = 32;     // per DP state front capacity
@@ -154,7 +158,38 @@ __device__ __forceinline__ void decode_vec(const DevParams &p, uint32_t B, uint3
 constexpr int kMS = 16;  // largest group on the split path
 constexpr int kH = 3;    // low members
 
-__device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, uint32_t B, int s, uint64_t v0,
+// Table accessors of the split evaluation (values widened to fp64 exactly;
+// dyn = fl(fl(p - P_s) * t) as in group64): straight from the staged fp32
+// blob, or from fp64 copies staged once per CTA in shared memory (no
+// per-use F2F conversion in the hot loops).
+struct Acc32 {
+  Tables tb;
+  double ps;
+  __device__ __forceinline__ double dd(int i) const { return (double)tb.d[i]; }
+  __device__ __forceinline__ double t(int r) const { return (double)tb.traw[r]; }
+  __device__ __forceinline__ double uu(int r) const { return (double)tb.u[r]; }
+  __device__ __forceinline__ double bb(int r) const { return (double)tb.bw[r]; }
+  __device__ __forceinline__ double dyn(int r) const {
+    return __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]);
+  }
+};
+struct Acc64 {
+  const double *d, *tt, *u, *bw, *dy;
+  __device__ __forceinline__ double dd(int i) const { return d[i]; }
+  __device__ __forceinline__ double t(int r) const { return tt[r]; }
+  __device__ __forceinline__ double uu(int r) const { return u[r]; }
+  __device__ __forceinline__ double bb(int r) const { return bw[r]; }
+  __device__ __forceinline__ double dyn(int r) const { return dy[r]; }
+};
+// fp64 shared-memory tables: d [R * ds] then t, u, bw, dyn [R] (R = n L rows)
+__host__ __device__ inline size_t acc64_bytes(const DevParams &p) {
+  const size_t R = (size_t)p.n * p.L;
+  return 8 * (R * p.ds + 4 * R);
+}
+constexpr size_t kAcc64Max = 40 << 10;  // staged only if it fits beside 4 CTAs per SM
+
+template <class A>
+__device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32_t B, int s, uint64_t v0,
                                          uint64_t v1, int lane, PPt *f, int &nf, bool &ok) {
   const int L = p.L, nh = s - kH;
   const uint32_t Lh = (uint32_t)(L * L * L);
@@ -186,9 +221,9 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
     for (int k = 0; k < kMS - kH; k++)
       if (k < nh) {
         const int r = rh[k];
-        U = __dadd_rn(U, (double)tb.u[r]);
-        Bw = __dadd_rn(Bw, (double)tb.bw[r]);
-        D = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]));
+        U = __dadd_rn(U, tb.uu(r));
+        Bw = __dadd_rn(Bw, tb.bb(r));
+        D = __dadd_rn(D, tb.dyn(r));
       }
 #pragma unroll
     for (int k = 0; k < kMS - kH; k++)
@@ -196,7 +231,7 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
         double a = 1.0;
 #pragma unroll
         for (int q = 0; q < kMS - kH; q++)
-          if (q < nh && q != k) a = __dadd_rn(a, (double)tb.d[rh[k] * p.ds + rh[q]]);
+          if (q < nh && q != k) a = __dadd_rn(a, tb.dd(rh[k] * p.ds + rh[q]));
         sg[k] = a;
       }
     double Q[kH][4];  // low member j at level l: 1 + sum over the high members
@@ -209,7 +244,7 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
           const int rj = mw[nh + j] * L + l;
 #pragma unroll
           for (int q = 0; q < kMS - kH; q++)
-            if (q < nh) a = __dadd_rn(a, (double)tb.d[rj * p.ds + rh[q]]);
+            if (q < nh) a = __dadd_rn(a, tb.dd(rj * p.ds + rh[q]));
         }
         Q[j][l] = a;
       }
@@ -223,27 +258,27 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
       const int r0b = mw[nh] * L, r1b = mw[nh + 1] * L, r2b = mw[nh + 2] * L;
       for (int d0 = 0; d0 < L; d0++) {
         const int r0 = r0b + d0;
-        const double U0 = __dadd_rn(U, (double)tb.u[r0]), B0 = __dadd_rn(Bw, (double)tb.bw[r0]);
-        const double D0 = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r0], ps), (double)tb.traw[r0]));
+        const double U0 = __dadd_rn(U, tb.uu(r0)), B0 = __dadd_rn(Bw, tb.bb(r0));
+        const double D0 = __dadd_rn(D, tb.dyn(r0));
         double a0[kMS - kH];
 #pragma unroll
         for (int k = 0; k < kMS - kH; k++)
-          if (k < nh) a0[k] = __dadd_rn(sg[k], (double)tb.d[rh[k] * p.ds + r0]);
+          if (k < nh) a0[k] = __dadd_rn(sg[k], tb.dd(rh[k] * p.ds + r0));
         for (int d1 = 0; d1 < L; d1++) {
           const int r1 = r1b + d1;
-          const double U1 = __dadd_rn(U0, (double)tb.u[r1]), B1 = __dadd_rn(B0, (double)tb.bw[r1]);
-          const double D1 = __dadd_rn(D0, __dmul_rn(__dsub_rn((double)tb.praw[r1], ps), (double)tb.traw[r1]));
+          const double U1 = __dadd_rn(U0, tb.uu(r1)), B1 = __dadd_rn(B0, tb.bb(r1));
+          const double D1 = __dadd_rn(D0, tb.dyn(r1));
           double a1[kMS - kH];
 #pragma unroll
           for (int k = 0; k < kMS - kH; k++)
-            if (k < nh) a1[k] = __dadd_rn(a0[k], (double)tb.d[rh[k] * p.ds + r1]);
-          const double s0p = __dadd_rn(Q[0][d0], (double)tb.d[r0 * p.ds + r1]);  // low 0: + low 1
-          const double s1p = __dadd_rn(Q[1][d1], (double)tb.d[r1 * p.ds + r0]);  // low 1: + low 0
+            if (k < nh) a1[k] = __dadd_rn(a0[k], tb.dd(rh[k] * p.ds + r1));
+          const double s0p = __dadd_rn(Q[0][d0], tb.dd(r0 * p.ds + r1));  // low 0: + low 1
+          const double s1p = __dadd_rn(Q[1][d1], tb.dd(r1 * p.ds + r0));  // low 1: + low 0
           for (int d2 = 0; d2 < L; d2++) {
             const int r2 = r2b + d2;
-            const double Ul = __dadd_rn(U1, (double)tb.u[r2]), Bl = __dadd_rn(B1, (double)tb.bw[r2]);
+            const double Ul = __dadd_rn(U1, tb.uu(r2)), Bl = __dadd_rn(B1, tb.bb(r2));
             const double Dl =
-                __dadd_rn(D1, __dmul_rn(__dsub_rn((double)tb.praw[r2], ps), (double)tb.traw[r2]));
+                __dadd_rn(D1, tb.dyn(r2));
             if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Ul > 1.0 || Bl > 1.0)) continue;
             double c = 1.0;
             if (Ul > c) c = Ul;
@@ -253,13 +288,13 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
             for (int k = 0; k < kMS - kH; k++)
               if (k < nh) {
                 const double ts =
-                    __dmul_rn((double)tb.traw[rh[k]], __dadd_rn(a1[k], (double)tb.d[rh[k] * p.ds + r2]));
+                    __dmul_rn(tb.t(rh[k]), __dadd_rn(a1[k], tb.dd(rh[k] * p.ds + r2)));
                 if (ts > mx) mx = ts;
               }
-            const double t0 = __dmul_rn((double)tb.traw[r0], __dadd_rn(s0p, (double)tb.d[r0 * p.ds + r2]));
-            const double t1 = __dmul_rn((double)tb.traw[r1], __dadd_rn(s1p, (double)tb.d[r1 * p.ds + r2]));
-            const double t2 = __dmul_rn((double)tb.traw[r2], __dadd_rn(__dadd_rn(Q[2][d2], (double)tb.d[r2 * p.ds + r0]),
-                                                                    (double)tb.d[r2 * p.ds + r1]));
+            const double t0 = __dmul_rn(tb.t(r0), __dadd_rn(s0p, tb.dd(r0 * p.ds + r2)));
+            const double t1 = __dmul_rn(tb.t(r1), __dadd_rn(s1p, tb.dd(r1 * p.ds + r2)));
+            const double t2 = __dmul_rn(tb.t(r2), __dadd_rn(__dadd_rn(Q[2][d2], tb.dd(r2 * p.ds + r0)),
+                                                                    tb.dd(r2 * p.ds + r1)));
             if (t0 > mx) mx = t0;
             if (t1 > mx) mx = t1;
             if (t2 > mx) mx = t2;
@@ -293,9 +328,9 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
       double Ul = U, Bl = Bw, Dl = D;
 #pragma unroll
       for (int j = 0; j < kH; j++) {
-        Ul = __dadd_rn(Ul, (double)tb.u[rl[j]]);
-        Bl = __dadd_rn(Bl, (double)tb.bw[rl[j]]);
-        Dl = __dadd_rn(Dl, __dmul_rn(__dsub_rn((double)tb.praw[rl[j]], ps), (double)tb.traw[rl[j]]));
+        Ul = __dadd_rn(Ul, tb.uu(rl[j]));
+        Bl = __dadd_rn(Bl, tb.bb(rl[j]));
+        Dl = __dadd_rn(Dl, tb.dyn(rl[j]));
       }
       if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Ul > 1.0 || Bl > 1.0)) continue;
       double c = 1.0;
@@ -308,8 +343,8 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
           double a = sg[k];
           const int rd = rh[k] * p.ds;
 #pragma unroll
-          for (int j = 0; j < kH; j++) a = __dadd_rn(a, (double)tb.d[rd + rl[j]]);
-          const double ts = __dmul_rn((double)tb.traw[rh[k]], a);
+          for (int j = 0; j < kH; j++) a = __dadd_rn(a, tb.dd(rd + rl[j]));
+          const double ts = __dmul_rn(tb.t(rh[k]), a);
           if (ts > mx) mx = ts;
         }
 #pragma unroll
@@ -317,8 +352,8 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
         double a = Q[j][dl[j]];
 #pragma unroll
         for (int j2 = 0; j2 < kH; j2++)
-          if (j2 != j) a = __dadd_rn(a, (double)tb.d[rl[j] * p.ds + rl[j2]]);
-        const double ts = __dmul_rn((double)tb.traw[rl[j]], a);
+          if (j2 != j) a = __dadd_rn(a, tb.dd(rl[j] * p.ds + rl[j2]));
+        const double ts = __dmul_rn(tb.t(rl[j]), a);
         if (ts > mx) mx = ts;
       }
       double Tg = __dmul_rn(mx, c);
@@ -337,11 +372,28 @@ __device__ __forceinline__ void pf_split(const Tables &tb, const DevParams &p, u
 }
 
 // phase 1a: work item = (group, 2^kItemLog2 level vectors); one warp per item
-__global__ void __launch_bounds__(256) k_pf_items(const DpParams dp) {
+__global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams dp) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, dp.p);
   const Tables tb = tables_at(sm, dp.p);
   const int lane = threadIdx.x & 31;
+  const bool use64 = dp.p.scope == SCHED_PER_CLIENT && acc64_bytes(dp.p) <= kAcc64Max;
+  Acc64 a64{};
+  if (use64) {
+    const int R = dp.p.n * dp.p.L;
+    double *b = (double *)(sm + ((dp.p.blob_bytes + 15) & ~15u));
+    double *rows = b + (size_t)R * dp.p.ds;
+    for (int i = threadIdx.x; i < R * dp.p.ds; i += blockDim.x) b[i] = (double)tb.d[i];
+    for (int r = threadIdx.x; r < R; r += blockDim.x) {
+      rows[r] = (double)tb.traw[r];
+      rows[R + r] = (double)tb.u[r];
+      rows[2 * R + r] = (double)tb.bw[r];
+      rows[3 * R + r] = __dmul_rn(__dsub_rn((double)tb.praw[r], dp.p.ps), (double)tb.traw[r]);
+    }
+    a64 = Acc64{b, rows, rows + R, rows + 2 * R, rows + 3 * R};
+    __syncthreads();
+  }
+  const Acc32 a32{tb, dp.p.ps};
   for (;;) {
     unsigned long long it = 0;
     if (lane == 0) it = atomicAdd(dp.ctr + kDpItem, 1ull);
@@ -365,7 +417,8 @@ __global__ void __launch_bounds__(256) k_pf_items(const DpParams dp) {
     bool ok = true;
     int lev[kMaxN];
     if (dp.p.scope == SCHED_PER_CLIENT && s > kH && s <= kMS && dp.p.L <= 4) {
-      pf_split(tb, dp.p, B, s, v0, v1, lane, f, nf, ok);
+      if (use64) pf_split(a64, dp.p, B, s, v0, v1, lane, f, nf, ok);
+      else pf_split(a32, dp.p, B, s, v0, v1, lane, f, nf, ok);
     } else {
       for (uint64_t v = v0 + lane; v < v1; v += 32) {
         decode_vec(dp.p, B, (uint32_t)v, lev);
@@ -750,7 +803,8 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
   CKD(cudaEventCreate(&e1));
   CKD(cudaEventRecord(e0, s));
   int nl = 0;
-  const size_t smem = (p.blob_bytes + 15) & ~15u;
+  const size_t smem = ((p.blob_bytes + 15) & ~15u) +
+                      (p.scope == SCHED_PER_CLIENT && acc64_bytes(p) <= kAcc64Max ? acc64_bytes(p) : 0);
   CKD(cudaFuncSetAttribute(k_pf_items, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   if (dp.nfull > 0) {
     k_pf_items<<<nsm * 4, 256, smem, s>>>(dp);
