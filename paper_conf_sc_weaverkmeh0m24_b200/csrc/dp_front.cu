@@ -204,6 +204,7 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       }
   }
   const double ps = p.ps;
+  double lt = __longlong_as_double(0x7ff0000000000000ll), le = lt;  // the lane's last inserted point
   for (uint64_t hv = v0 / Lh + lane; hv * Lh < v1; hv += 32) {
     int rh[kMS - kH];
     double sg[kMS - kH];
@@ -308,7 +309,12 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
             x.e = __dadd_rn(__dmul_rn(ps, Tg), Dl);
             x.v = (uint32_t)(base + (uint32_t)((d0 * L + d1) * L + d2));
             x.pad = 0;
+            // quick reject: a point inserted earlier (lt, le) dominates or equals x ->
+            // so does the front (transitivity), front_insert would keep it unchanged
+            if (x.t >= lt && x.e >= le) continue;
             ok &= front_insert<kLF>(f, nf, x);
+            lt = x.t;
+            le = x.e;
           }
         }
       }

@@ -1,5 +1,5 @@
 # subset-DP phase 1 with fp64 shared-memory tables: register budget variants
-for v in "-DSCHED_PF_MINB=1" "-DSCHED_PF_MINB=2"; do
+for v in ""; do
   rm -f paper_conf_sc_weaverkmeh0m24_b200/build_obj/dp_front* paper_conf_sc_weaverkmeh0m24_b200/libsched.so
   SCHED_NVCC_EXTRA="$v" python -c "import __graft_entry__ as g; g.build()" 2>&1 | tail -1
   echo "variant [$v]"
