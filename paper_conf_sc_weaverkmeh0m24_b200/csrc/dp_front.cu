@@ -214,8 +214,8 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
 #pragma unroll
       for (int k = kMS - kH - 1; k >= 0; k--)
         if (k < nh) {
-          rh[k] = mw[k] * L + (int)(x % (uint64_t)L);
-          x /= (uint64_t)L;
+          rh[k] = mw[k] * L + (int)((uint32_t)x % (uint32_t)L);  // hv < 4^13: 32-bit
+          x = (uint32_t)x / (uint32_t)L;
         }
     }
 #pragma unroll

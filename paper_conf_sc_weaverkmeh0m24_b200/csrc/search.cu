@@ -28,9 +28,23 @@ __device__ __forceinline__ void decode_levels(const DevParams &p, const LaneCfg 
   const int nd = p.scope == SCHED_PER_CLIENT ? p.n : c.k;
   int dig[kMaxN];
   u64 x = c.v;
-  for (int d = nd - 1; d >= 0; d--) {
-    dig[d] = (int)(x % (u64)p.L);
-    x /= (u64)p.L;
+  if ((p.L & (p.L - 1)) == 0) {  // L = 1, 2, 4, 8: shifts (a u64 division is ~100 instructions)
+    const int sh = __ffs(p.L) - 1;
+    for (int d = nd - 1; d >= 0; d--) {
+      dig[d] = (int)(x & (u64)(p.L - 1));
+      x >>= sh;
+    }
+  } else if (x <= 0xffffffffull) {  // 32-bit division
+    uint32_t y = (uint32_t)x;
+    for (int d = nd - 1; d >= 0; d--) {
+      dig[d] = (int)(y % (uint32_t)p.L);
+      y /= (uint32_t)p.L;
+    }
+  } else {
+    for (int d = nd - 1; d >= 0; d--) {
+      dig[d] = (int)(x % (u64)p.L);
+      x /= (u64)p.L;
+    }
   }
   for (int i = 0; i < p.n; i++) lam[i] = p.scope == SCHED_PER_CLIENT ? dig[i] : dig[c.a[i]];
 }
