@@ -1,7 +1,7 @@
 // search.cu -- the exhaustive configuration search on sm_100a.
 //
 //   k_generic   any scope / L / G / C / weights: per-lane unrank + successor
-//               walk, from-scratch fp32 group scoring, fp32 screens, fp64
+//               walk, incremental fp32 group scoring, fp32 screens, fp64
 //               canonical refine of near-best / possibly-Pareto configurations.
 //   k_best_final, k_pareto_* : per-GPU finalize (exact best, exact Pareto).
 //
@@ -49,13 +49,32 @@ __device__ __forceinline__ void decode_levels(const DevParams &p, const LaneCfg 
   for (int i = 0; i < p.n; i++) lam[i] = p.scope == SCHED_PER_CLIENT ? dig[i] : dig[c.a[i]];
 }
 
-// fp32 score, normalised: returns T/T_seq and E/E_seq (hot-loop precision)
-__device__ __forceinline__ void score32(const Tables &tb, const DevParams &p, const LaneCfg &c,
-                                        const int *lam, float &T, float &E) {
-  T = 0.f;
-  E = 0.f;
-  float Dall = 0.f;
-  for (int g = 0; g < c.k; g++) {
+// fp32 score, normalised (hot-loop precision): T/T_seq and E/E_seq of the
+// lane's configuration, per group U, B, D (members ascending), c_g, sigma_i,
+// T_g = max_i t_i sigma_i c_g; T = max_g T_g, E = sum_g (P_s T_g + D_g) in
+// group order.  Incremental over the successor walk: the per-group terms
+// (T_g, P_s T_g + D_g, D_g) of the lane's current partition are cached and
+// only the groups holding a client whose level changed (or every group after
+// a partition change) are re-scored -- the same per-group operations and the
+// same group-order combination as a from-scratch evaluation, hence the same
+// fp32 values.
+struct GroupCache {
+  float t[kMaxG], e[kMaxG], d[kMaxG];
+  int lam[kMaxN];
+  bool valid;
+};
+
+__device__ __forceinline__ void score32_inc(const Tables &tb, const DevParams &p, const LaneCfg &c,
+                                            const int *lam, GroupCache &gc, float &T, float &E) {
+  uint32_t dirty = 0;
+  if (!gc.valid) {
+    dirty = c.k >= 32 ? 0xffffffffu : (1u << c.k) - 1;
+  } else {
+    for (int i = 0; i < p.n; i++)
+      if (lam[i] != gc.lam[i]) dirty |= 1u << c.a[i];
+  }
+  for (uint32_t dd = dirty; dd; dd &= dd - 1) {
+    const int g = __ffs(dd) - 1;
     const uint32_t m = c.mask[g];
     float U = 0.f, B = 0.f, D = 0.f;
     for (uint32_t mm = m; mm; mm &= mm - 1) {
@@ -73,9 +92,19 @@ __device__ __forceinline__ void score32(const Tables &tb, const DevParams &p, co
       Tg = fmaxf(Tg, tb.th[ri] * s * cg);
     }
     if (p.model & SCHED_MODEL_POWER_CAP) Tg = fmaxf(Tg, D * p.kcap);  // R28
-    T = fmaxf(T, Tg);
-    E += p.phat * Tg + D;
-    Dall += D;
+    gc.t[g] = Tg;
+    gc.e[g] = p.phat * Tg + D;
+    gc.d[g] = D;
+  }
+  for (int i = 0; i < p.n; i++) gc.lam[i] = lam[i];
+  gc.valid = true;
+  T = 0.f;
+  E = 0.f;
+  float Dall = 0.f;
+  for (int g = 0; g < c.k; g++) {
+    T = fmaxf(T, gc.t[g]);
+    E += gc.e[g];
+    Dall += gc.d[g];
   }
   if (p.model & SCHED_MODEL_COUNT_IDLE) E = p.kidle * T + Dall;  // R26
 }
@@ -114,6 +143,7 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
   const int ul = p.unit_log2, cl = p.chunk_log2;
   LaneCfg c;
   int lam[kMaxN];
+  GroupCache gc;
 
   for (;;) {
     u64 unit = 0;
@@ -141,6 +171,7 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
     const u64 lend = p.lane_strided ? e : (idx + run < e ? idx + run : e);
     const u64 step = p.lane_strided ? 32 : 1;
     if (idx < lend && dev_unrank(tb, p, idx, c)) {
+      gc.valid = false;
       for (;;) {
         ncfg++;
         bool feas = c.feasible;
@@ -152,7 +183,7 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
           nfeas++;
           decode_levels(p, c, lam);
           float T, E;
-          score32(tb, p, c, lam, T, E);
+          score32_inc(tb, p, c, lam, gc, T, E);
           bool need = false;
           unsigned wneed = 0;
 #pragma unroll
@@ -196,6 +227,7 @@ __global__ void __launch_bounds__(kThreads) k_generic(const DevParams p) {
         }
         idx += step;
         if (idx >= lend) break;
+        if (c.v + step >= c.Pn) gc.valid = false;  // the successor walk leaves the partition
         if (!dev_advance(tb, p, c, step)) break;
       }
     }
