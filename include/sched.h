@@ -141,7 +141,8 @@ typedef struct {
   double t_seq_s, e_seq_j;      /* sequential baselines */
   float search_ms;              /* device time of the search kernel(s) (CUDA events) */
   float total_ms;               /* device time of the whole call on the stream */
-  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile, 2 L=1 pair, 3 L=1 suffix, 4 subset-DP front */
+  int32_t kernel_path;          /* 0 generic, 1 PER_GPU tile, 2 L=1 pair, 3 L=1 suffix, 4 subset-DP front,
+                                   5 PER_CLIENT tile */
   int32_t grid_ctas;            /* persistent CTAs launched by the search kernel */
   int32_t kernel_launches;      /* kernels this call launched (init, search pass(es), finalize) */
   int32_t passes;               /* search passes (2 = re-run after candidate overflow) */

@@ -1,0 +1,45 @@
+// ctile.cu -- eligibility and launch of the PER_CLIENT tile kernel
+// (search_ctile.cuh): PER_CLIENT scope, L = 4, 6 <= n <= 15, canonical model
+// or POWER_CAP (E = sum_g E_g, level-independent feasibility).
+#include "search_ctile.cuh"
+
+namespace sched {
+
+static size_t ctile_smem(const DevParams &dp) {
+  return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(CtWarp) * kCtWarps + sizeof(BestRec) * kCtWarps * kMaxW;
+}
+
+bool ctile_eligible(DevParams &dp, TileLaunch *tl) {
+  if (dp.scope != SCHED_PER_CLIENT || dp.L != 4 || dp.n < 6 || dp.n > 15) return false;
+  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE)) return false;
+  tl->fn = (const void *)k_ctile;
+  tl->smem = ctile_smem(dp);
+  return true;
+}
+
+cudaError_t launch_ctile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                         cudaEvent_t e2, int *grid, bool fixed_units) {
+  cudaError_t err = cudaFuncSetAttribute(tl.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tl.smem);
+  if (err != cudaSuccess) return err;
+  int occ = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kCtThreads, tl.smem);
+  if (err != cudaSuccess) return err;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  *grid = std::min(4096, nsm * occ);
+  if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
+    const uint64_t range = dp.n_owned << dp.chunk_log2;
+    const uint64_t warps = (uint64_t)(*grid) * kCtWarps;
+    int ul = 12;
+    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 8) ul++;
+    dp.unit_log2 = ul;
+    dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+    dp.unit_stride = 1;
+  }
+  void *args[] = {(void *)&dp};
+  cudaEventRecord(e1, st);
+  err = cudaLaunchKernel(tl.fn, *grid, kCtThreads, args, tl.smem, st);
+  cudaEventRecord(e2, st);
+  return err;
+}
+
+}  // namespace sched

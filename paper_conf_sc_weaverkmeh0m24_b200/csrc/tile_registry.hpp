@@ -40,6 +40,9 @@ size_t tile_smem_bytes(const DevParams &dp);
 bool tile_eligible(DevParams &dp, TileLaunch *tl);
 bool dfs_eligible(DevParams &dp, TileLaunch *tl);
 bool sfx_eligible(DevParams &dp, TileLaunch *tl);
+bool ctile_eligible(DevParams &dp, TileLaunch *tl);
+cudaError_t launch_ctile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                         cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
                        cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_dfs(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,

@@ -273,3 +273,25 @@ def test_maximum_sizes_windows(n, g, c, levels, scope):
     for lo in (0, tot // 3 + 12345, tot - 150_000):
         qw = q.with_range(lo, min(tot, lo + 150_000))
         check(sch.search(qw), oracle.search(prof, qw), qw)
+
+
+@pytest.mark.parametrize("n,g,c,ws,pareto,model,seed", [
+    (6, 3, 3, ((1, 0), (0, 1), (1, 1), (2, 1)), True, 0, 11),
+    (6, 2, 6, ((1, 1),), True, 4, 12),                 # POWER_CAP variant
+    (7, 4, 7, ((1, 0),), False, 0, 13),
+    (7, 4, 2, ((2, 1), (1, 3)), True, 0, 14),
+    (6, 6, 6, (), True, 0, 15),                        # Pareto only, many groups
+])
+def test_client_tile_kernel_path(n, g, c, ws, pareto, model, seed):
+    """PER_CLIENT, L = 4 spaces on the PER_CLIENT tile kernel (kernel_path 5):
+    full space and ragged windows bitwise against the oracle."""
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, (25, 50, 75, 100), PER_CLIENT, ws, pareto, model=model, power_cap=150.0)
+    sch = S.Scheduler(prof)
+    res = sch.search(q)
+    assert res.stats["kernel_path"] == 5
+    check(res, oracle.search(prof, q), q)
+    tot = S.count(q)
+    for lo, hi in ((1000, 70_001), (tot // 2 - 4097, tot // 2 + 33_333), (tot - 50_000, tot)):
+        qw = q.with_range(lo, hi)
+        check(sch.search(qw), oracle.search(prof, qw), qw)
