@@ -31,13 +31,14 @@ struct CtWarp {
   u64 base;
 };
 
-// fp32 normalised (T_g, E-term) of group m at the lane's levels lam[]
-// (the per-group operations of the generic kernel's score32_inc)
-__device__ __forceinline__ void ct_group32(const Tables &tb, const DevParams &p, uint32_t m, const int *lam,
+// fp32 normalised (T_g, E-term) of group m at the levels packed in lw
+// (2 bits per client: register-resident, no local-memory level array; the
+// per-group operations of the generic kernel's score32_inc)
+__device__ __forceinline__ void ct_group32(const Tables &tb, const DevParams &p, uint32_t m, uint32_t lw,
                                            float &Tg, float &Eg) {
   float U = 0.f, B = 0.f, D = 0.f;
   for (uint32_t mm = m; mm; mm &= mm - 1) {
-    const int i = __ffs(mm) - 1, r = i * 4 + lam[i];
+    const int i = __ffs(mm) - 1, r = i * 4 + (int)((lw >> (2 * i)) & 3u);
     U += tb.u[r];
     B += tb.bw[r];
     D += tb.dh[r];
@@ -45,9 +46,12 @@ __device__ __forceinline__ void ct_group32(const Tables &tb, const DevParams &p,
   const float cg = fmaxf(fmaxf(1.f, U), B);
   float T = 0.f;
   for (uint32_t mm = m; mm; mm &= mm - 1) {
-    const int i = __ffs(mm) - 1, ri = i * 4 + lam[i];
+    const int i = __ffs(mm) - 1, ri = i * 4 + (int)((lw >> (2 * i)) & 3u);
     float s = 1.f;
-    for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) s += tb.d[ri * p.ds + (__ffs(m2) - 1) * 4 + lam[__ffs(m2) - 1]];
+    for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) {
+      const int j = __ffs(m2) - 1;
+      s += tb.d[ri * p.ds + j * 4 + (int)((lw >> (2 * j)) & 3u)];
+    }
     T = fmaxf(T, tb.th[ri] * s * cg);
   }
   if (p.model & SCHED_MODEL_POWER_CAP) T = fmaxf(T, D * p.kcap);  // R28
@@ -55,9 +59,18 @@ __device__ __forceinline__ void ct_group32(const Tables &tb, const DevParams &p,
   Eg = p.phat * T + D;
 }
 
+__device__ __forceinline__ uint32_t ct_set(uint32_t lw, int x, int l) {
+  return (lw & ~(3u << (2 * x))) | ((uint32_t)l << (2 * x));
+}
+
 // exact canonical fp64 (T_g, E_g) of group m (refine64 for one group)
-__device__ __forceinline__ void ct_group64(const Tables &tb, const DevParams &p, uint32_t m, const int *lam,
+__device__ __forceinline__ void ct_group64(const Tables &tb, const DevParams &p, uint32_t m, uint32_t lw,
                                            double &Tg, double &Eg) {
+  int lam[kMaxN];
+  for (uint32_t mm = m; mm; mm &= mm - 1) {
+    const int i = __ffs(mm) - 1;
+    lam[i] = (int)((lw >> (2 * i)) & 3u);
+  }
   refine64(tb, p, &m, 1, lam, &Tg, &Eg);
 }
 
@@ -116,11 +129,15 @@ __device__ __noinline__ int ct_edge(const Tables &tb, const DevParams &p, const 
   int nref = 0;
   int lam[kMaxN];
   for (uint32_t v = v0; v < v1; v += step) {
-    for (int i = 0; i < n; i++) lam[i] = (int)(v >> (2 * (n - 1 - i))) & 3;
+    uint32_t lw = 0;
+    for (int i = 0; i < n; i++) {
+      lam[i] = (int)(v >> (2 * (n - 1 - i))) & 3;
+      lw |= (uint32_t)lam[i] << (2 * i);
+    }
     float T = 0.f, E = 0.f;
     for (int g = 0; g < k; g++) {
       float Tg, Eg;
-      ct_group32(tb, p, wp.cfg.mask[g], lam, Tg, Eg);
+      ct_group32(tb, p, wp.cfg.mask[g], lw, Tg, Eg);
       T = fmaxf(T, Tg);
       E += Eg;
     }
@@ -202,18 +219,16 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
           const uint32_t tbits = (3u << s1) | (3u << s2) | (3u << s3);
           for (uint32_t o = lane; o < nout; o += 32) {
             // outer string o -> levels of the non-tile clients (ascending, most significant first)
-            int lam[kMaxN];
+            uint32_t lw = 0;  // levels, 2 bits per client (tile clients 0)
             uint32_t vo = 0;  // the outer digits' contribution to the level-vector index
             {
               int sh = 2 * (n - 4);
               for (int i = 0; i < n; i++) {
-                if (tmask >> i & 1u) {
-                  lam[i] = 0;
-                  continue;
-                }
-                lam[i] = (int)(o >> sh) & 3;
+                if (tmask >> i & 1u) continue;
+                const uint32_t d = (o >> sh) & 3u;
                 sh -= 2;
-                vo |= (uint32_t)lam[i] << (2 * (n - 1 - i));
+                lw |= d << (2 * i);
+                vo |= d << (2 * (n - 1 - i));
               }
             }
             // the tile's index span [vo, vo | tbits]: skip it if it misses [v0, v1)
@@ -222,19 +237,17 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
             float Tp = 0.f, Ep = 0.f;
             for (int g = 0; g < k - 3; g++) {
               float Tg, Eg;
-              ct_group32(tb, p, wp.cfg.mask[g], lam, Tg, Eg);
+              ct_group32(tb, p, wp.cfg.mask[g], lw, Tg, Eg);
               Tp = fmaxf(Tp, Tg);
               Ep += Eg;
             }
             float At[4], Ae[4], Bt[4], Be[4], Ct[4], Ce[4];
 #pragma unroll
             for (int l = 0; l < 4; l++) {
-              lam[x1] = l;
-              lam[x2] = l;
-              lam[x3] = l;
-              ct_group32(tb, p, ma, lam, At[l], Ae[l]);
-              ct_group32(tb, p, mb, lam, Bt[l], Be[l]);
-              ct_group32(tb, p, mc, lam, Ct[l], Ce[l]);
+              const uint32_t ll = ct_set(ct_set(ct_set(lw, x1, l), x2, l), x3, l);
+              ct_group32(tb, p, ma, ll, At[l], Ae[l]);
+              ct_group32(tb, p, mb, ll, Bt[l], Be[l]);
+              ct_group32(tb, p, mc, ll, Ct[l], Ce[l]);
             }
             if (whole) {
               // the tile's 64 configurations, min-reduced to the exact lower corner
@@ -270,18 +283,16 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
             double Tp64 = 0.0, Ep64 = 0.0;
             for (int g = 0; g < k - 3; g++) {
               double Tg, Eg;
-              ct_group64(tb, p, wp.cfg.mask[g], lam, Tg, Eg);
+              ct_group64(tb, p, wp.cfg.mask[g], lw, Tg, Eg);
               if (Tg > Tp64) Tp64 = Tg;
               Ep64 = __dadd_rn(Ep64, Eg);
             }
             double A64[4], AE64[4], B64[4], BE64[4], C64[4], CE64[4];
             for (int l = 0; l < 4; l++) {
-              lam[x1] = l;
-              lam[x2] = l;
-              lam[x3] = l;
-              ct_group64(tb, p, ma, lam, A64[l], AE64[l]);
-              ct_group64(tb, p, mb, lam, B64[l], BE64[l]);
-              ct_group64(tb, p, mc, lam, C64[l], CE64[l]);
+              const uint32_t ll = ct_set(ct_set(ct_set(lw, x1, l), x2, l), x3, l);
+              ct_group64(tb, p, ma, ll, A64[l], AE64[l]);
+              ct_group64(tb, p, mb, ll, B64[l], BE64[l]);
+              ct_group64(tb, p, mc, ll, C64[l], CE64[l]);
             }
             for (int a = 0; a < 4; a++)
               for (int b = 0; b < 4; b++)
