@@ -76,12 +76,12 @@ __device__ __forceinline__ void ct_group64(const Tables &tb, const DevParams &p,
 
 // One configuration with known fp32 (T, E) and a way to get its exact fp64
 // (T, E): weight screens (lane thresholds), Pareto screen, fp64 record.
-template <class Exact>
+template <int WM, class Exact>
 __device__ __forceinline__ int ct_check(const DevParams &p, const Stair &stair, float *thr, BestRec *lb, u64 idx,
                                         float T, float E, Exact exact) {
   unsigned need = 0;
 #pragma unroll
-  for (int w = 0; w < kMaxW; w++) {
+  for (int w = 0; w < WM; w++) {
     if (w < p.nw) {
       float q = 1.f;
       for (int i = 0; i < p.wa[w]; i++) q *= T;
@@ -101,7 +101,7 @@ __device__ __forceinline__ int ct_check(const DevParams &p, const Stair &stair, 
   if (!need && !par) return 0;
   if (!have) exact(T64, E64);
 #pragma unroll
-  for (int w = 0; w < kMaxW; w++) {
+  for (int w = 0; w < WM; w++) {
     if (need >> w & 1u) {
       const double F = objective64(p, T64, E64, p.wa[w], p.wb[w]);
       if (!lb[w].valid || better(F, idx, lb[w].f, lb[w].idx)) {
@@ -123,6 +123,7 @@ __device__ __forceinline__ int ct_check(const DevParams &p, const Stair &stair, 
 
 // Per-configuration path: level vectors v in [v0, v1) step `step` of the
 // partition (from-scratch fp32 score, refine64 when screened in).
+template <int WM>
 __device__ __noinline__ int ct_edge(const Tables &tb, const DevParams &p, const Stair &stair, const CtWarp &wp,
                                     float *thr, BestRec *lb, uint32_t v0, uint32_t v1, uint32_t step) {
   const int n = p.n, k = wp.cfg.k;
@@ -141,13 +142,16 @@ __device__ __noinline__ int ct_edge(const Tables &tb, const DevParams &p, const 
       T = fmaxf(T, Tg);
       E += Eg;
     }
-    nref += ct_check(p, stair, thr, lb, wp.base + v, T, E, [&](double &T64, double &E64) {
+    nref += ct_check<WM>(p, stair, thr, lb, wp.base + v, T, E, [&](double &T64, double &E64) {
       refine64(tb, p, wp.cfg.mask, k, lam, &T64, &E64);
     });
   }
   return nref;
 }
 
+// WM: weights held per lane (thresholds, best records) -- the smallest of
+// 1, 2, 4, 8 that covers the query, to keep the per-thread stack small
+template <int WM>
 __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, p);
@@ -161,10 +165,10 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
   stair_init(stair);
   __syncthreads();
 
-  float thr[kMaxW];
-  BestRec lb[kMaxW];
+  float thr[WM];
+  BestRec lb[WM];
 #pragma unroll
-  for (int w = 0; w < kMaxW; w++) {
+  for (int w = 0; w < WM; w++) {
     thr[w] = __int_as_float(0x7f800000);
     best_init(lb[w]);
   }
@@ -187,7 +191,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
     e = e < p.hi ? e : p.hi;
     if (s >= e) continue;
 #pragma unroll
-    for (int w = 0; w < kMaxW; w++)
+    for (int w = 0; w < WM; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
     if (p.want_pareto) stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     if (lane == 0) {
@@ -209,7 +213,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
       }
       if (feas) {
         if (k < 3) {
-          nref += ct_edge(tb, p, stair, wp, thr, lb, v0 + lane, v1, 32);
+          nref += ct_edge<WM>(tb, p, stair, wp, thr, lb, v0 + lane, v1, 32);
         } else {
           // tile clients: the highest member of each of the last three blocks
           const uint32_t ma = wp.cfg.mask[k - 3], mb = wp.cfg.mask[k - 2], mc = wp.cfg.mask[k - 1];
@@ -267,7 +271,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
               }
               bool hit = false;
 #pragma unroll
-              for (int w = 0; w < kMaxW; w++) {
+              for (int w = 0; w < WM; w++) {
                 if (w < p.nw) {
                   float q = 1.f;
                   for (int i = 0; i < p.wa[w]; i++) q *= mT;
@@ -301,7 +305,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
                   if (v < v0 || v >= v1) continue;
                   const float T = fmaxf(fmaxf(fmaxf(Tp, At[a]), Bt[b]), Ct[c]);
                   const float E = ((Ep + Ae[a]) + Be[b]) + Ce[c];
-                  nref += ct_check(p, stair, thr, lb, base + v, T, E, [&](double &T64, double &E64) {
+                  nref += ct_check<WM>(p, stair, thr, lb, base + v, T, E, [&](double &T64, double &E64) {
                     T64 = fmax(fmax(fmax(Tp64, A64[a]), B64[b]), C64[c]);
                     E64 = __dadd_rn(__dadd_rn(__dadd_rn(Ep64, AE64[a]), BE64[b]), CE64[c]);
                   });
@@ -321,7 +325,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
       __syncwarp();
     }
 #pragma unroll
-    for (int w = 0; w < kMaxW; w++) {
+    for (int w = 0; w < WM; w++) {
       if (w < p.nw) {
         float t = thr[w];
 #pragma unroll
@@ -344,7 +348,7 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
     atomicAdd(p.ctr + kCtrRefined, nref64);
   }
 #pragma unroll
-  for (int w = 0; w < kMaxW; w++) {
+  for (int w = 0; w < WM; w++) {
     if (w < p.nw) {
       warp_best(lb[w]);
       if (lane == 0) red[warp * kMaxW + w] = lb[w];
@@ -360,6 +364,11 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
     }
     ((BestRec *)p.slots)[(size_t)blockIdx.x * p.nw + w] = b;
   }
+}
+
+template <int WM>
+const void *ctile_fn() {
+  return (const void *)k_ctile<WM>;
 }
 
 }  // namespace sched
