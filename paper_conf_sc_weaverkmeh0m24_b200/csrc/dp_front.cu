@@ -261,10 +261,6 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
         const int r0 = r0b + d0;
         const double U0 = __dadd_rn(U, tb.uu(r0)), B0 = __dadd_rn(Bw, tb.bb(r0));
         const double D0 = __dadd_rn(D, tb.dyn(r0));
-        double a0[kMS - kH];
-#pragma unroll
-        for (int k = 0; k < kMS - kH; k++)
-          if (k < nh) a0[k] = __dadd_rn(sg[k], tb.dd(rh[k] * p.ds + r0));
         for (int d1 = 0; d1 < L; d1++) {
           const int r1 = r1b + d1;
           const double U1 = __dadd_rn(U0, tb.uu(r1)), B1 = __dadd_rn(B0, tb.bb(r1));
@@ -272,7 +268,8 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
           double a1[kMS - kH];
 #pragma unroll
           for (int k = 0; k < kMS - kH; k++)
-            if (k < nh) a1[k] = __dadd_rn(a0[k], tb.dd(rh[k] * p.ds + r1));
+            if (k < nh)  // (sg + d[k][low 0]) + d[k][low 1]: the a0 partial re-formed per d1 (fewer live registers)
+              a1[k] = __dadd_rn(__dadd_rn(sg[k], tb.dd(rh[k] * p.ds + r0)), tb.dd(rh[k] * p.ds + r1));
           const double s0p = __dadd_rn(Q[0][d0], tb.dd(r0 * p.ds + r1));  // low 0: + low 1
           const double s1p = __dadd_rn(Q[1][d1], tb.dd(r1 * p.ds + r0));  // low 1: + low 0
           for (int d2 = 0; d2 < L; d2++) {
