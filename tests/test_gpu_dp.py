@@ -105,3 +105,20 @@ def test_dp_front_c4_client_prefix_golden(n):
     assert [b.score64.hex() for b in best] == g["best_score64"]
     for x in list(front) + list(best):
         assert _witness_ok(p, q, x)
+
+
+def test_dp_front_c5_equals_certificate():
+    """c5 (20 workflows, 8 GPUs, <= 3 clients per GPU, 6.0e11 configurations):
+    the device DP front and the 7-weight sweep optimum equal the stored O3
+    certificate bitwise (tests/golden/c5_certificate.json)."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c5_certificate.json")))
+    prof, q = config("c5")
+    rc, best, front, st = S.Scheduler(prof).front_dp(q)
+    assert rc == S.sched.SCHED_OK and st["kernel_path"] == 4
+    assert [[p.makespan_s.hex(), p.energy_j.hex()] for p in front] == g["front_T_E"]
+    assert [b.score64.hex() for b in best] == g["best_score64"]
+    for p in list(front) + list(best):
+        assert _witness_ok(prof, q, p)
+    print("c5 DP:", st["total_ms"], "ms")
