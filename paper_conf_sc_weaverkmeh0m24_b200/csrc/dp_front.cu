@@ -257,6 +257,75 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       // a deeper low member is formed once at its loop level -- the same
       // additions in the same ascending-member order as below.
       const int r0b = mw[nh] * L, r1b = mw[nh + 1] * L, r2b = mw[nh + 2] * L;
+      if (nf > 0) {
+        // Block lower corner: every canonical sum with each low member's term
+        // replaced by its minimum over the levels (same order; rounding is
+        // monotone, all terms >= 0), so T >= Tmin and E >= Emin for every
+        // vector of the block.  A front point at or below the corner
+        // dominates (or equals) all 64 vectors: skip the block.
+        const int rb[kH] = {r0b, r1b, r2b};
+        double Umin = U, Bmin = Bw, Dmin = D;
+#pragma unroll
+        for (int j = 0; j < kH; j++) {
+          double um = tb.uu(rb[j]), bm = tb.bb(rb[j]), dm = tb.dyn(rb[j]);
+          for (int l = 1; l < L; l++) {
+            um = fmin(um, tb.uu(rb[j] + l));
+            bm = fmin(bm, tb.bb(rb[j] + l));
+            dm = fmin(dm, tb.dyn(rb[j] + l));
+          }
+          Umin = __dadd_rn(Umin, um);
+          Bmin = __dadd_rn(Bmin, bm);
+          Dmin = __dadd_rn(Dmin, dm);
+        }
+        if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Umin > 1.0 || Bmin > 1.0)) continue;  // all infeasible
+        double cmin = 1.0;
+        if (Umin > cmin) cmin = Umin;
+        if (Bmin > cmin) cmin = Bmin;
+        double mx = 0.0;
+#pragma unroll
+        for (int k = 0; k < kMS - kH; k++)
+          if (k < nh) {
+            double a = sg[k];
+#pragma unroll
+            for (int j = 0; j < kH; j++) {
+              double dmn = tb.dd(rh[k] * p.ds + rb[j]);
+              for (int l = 1; l < L; l++) dmn = fmin(dmn, tb.dd(rh[k] * p.ds + rb[j] + l));
+              a = __dadd_rn(a, dmn);
+            }
+            const double ts = __dmul_rn(tb.t(rh[k]), a);
+            if (ts > mx) mx = ts;
+          }
+#pragma unroll
+        for (int j = 0; j < kH; j++) {
+          double tj = 0.0;  // min over the member's own level of its bound
+          for (int l = 0; l < L; l++) {
+            double a = Q[j][l];
+#pragma unroll
+            for (int j2 = 0; j2 < kH; j2++)
+              if (j2 != j) {
+                double dmn = tb.dd((rb[j] + l) * p.ds + rb[j2]);
+                for (int l2 = 1; l2 < L; l2++) dmn = fmin(dmn, tb.dd((rb[j] + l) * p.ds + rb[j2] + l2));
+                a = __dadd_rn(a, dmn);
+              }
+            const double ts = __dmul_rn(tb.t(rb[j] + l), a);
+            tj = l == 0 ? ts : fmin(tj, ts);
+          }
+          if (tj > mx) mx = tj;
+        }
+        double Tmin = __dmul_rn(mx, cmin);
+        if (p.model & SCHED_MODEL_POWER_CAP) {
+          const double tcap = __ddiv_rn(Dmin, p.capd);
+          if (tcap > Tmin) Tmin = tcap;
+        }
+        const double Emin = __dadd_rn(__dmul_rn(ps, Tmin), Dmin);
+        bool skip = false;
+        for (int i = 0; i < nf; i++)
+          if (f[i].t <= Tmin && f[i].e <= Emin) {
+            skip = true;
+            break;
+          }
+        if (skip) continue;
+      }
       for (int d0 = 0; d0 < L; d0++) {
         const int r0 = r0b + d0;
         const double U0 = __dadd_rn(U, tb.uu(r0)), B0 = __dadd_rn(Bw, tb.bb(r0));
