@@ -295,3 +295,44 @@ def test_client_tile_kernel_path(n, g, c, ws, pareto, model, seed):
     for lo, hi in ((1000, 70_001), (tot // 2 - 4097, tot // 2 + 33_333), (tot - 50_000, tot)):
         qw = q.with_range(lo, hi)
         check(sch.search(qw), oracle.search(prof, qw), qw)
+
+
+def test_bench_slice_launch_configuration():
+    """One bench.py step exactly as it is timed (c4, shard (sigma, 64) of
+    2^22-index chunks, 3.2e12 configurations): coverage equals the slice's
+    index count, every returned configuration re-scores bitwise in the
+    oracle, the slice's optimum never beats the O3 certificate's, and no
+    sampled oracle window of the slice beats the slice's best or escapes its
+    Pareto front."""
+    import json
+    import os
+    prof, q = config("c4")
+    sigma, slices, cl = 5, 64, 22
+    tot = S.count(q)
+    sch = S.Scheduler(prof)
+    res = sch.search(q, shard=(sigma, slices), chunk_log2=cl)
+    nch = (tot + (1 << cl) - 1) >> cl
+    want = sum(min(tot, (c + 1) << cl) - (c << cl) for c in range(sigma, nch, slices))
+    assert res.stats["n_configs"] == want
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c4_certificate.json")))
+    for w, b in enumerate(res.best):
+        assert b.valid and (b.index >> cl) % slices == sigma
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, b.index))
+        assert ok and (T, E) == (b.makespan_s, b.energy_j)
+        assert b.score64 <= float.fromhex(g["best_score64"][w])
+    for p in res.pareto:
+        assert (p.index >> cl) % slices == sigma
+        ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
+        assert ok and (T, E) == (p.makespan_s, p.energy_j)
+    front = [(p.makespan_s, p.energy_j) for p in res.pareto]
+    rnd = random.Random(17)
+    for _ in range(4):
+        c = sigma + slices * rnd.randrange((nch - sigma) // slices - 1)  # whole chunks only
+        lo = (c << cl) + rnd.randrange((1 << cl) - 200_000)
+        r = oracle.search(prof, q.with_range(lo, lo + 200_000))
+        for w, b in enumerate(res.best):
+            x = r["best"][w]
+            if x is not None:
+                assert x[1] < b.score64 or (x[1] == b.score64 and x[0] >= b.index)
+        for _, T, E in r["pareto"]:
+            assert any(t2 <= T and e2 <= E for t2, e2 in front)
