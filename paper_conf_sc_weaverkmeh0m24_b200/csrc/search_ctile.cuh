@@ -59,6 +59,61 @@ __device__ __forceinline__ void ct_group32(const Tables &tb, const DevParams &p,
   Eg = p.phat * T + D;
 }
 
+// The same fp32 group values at the 4 levels of the group's HIGHEST member
+// x (the tile client): x's terms come last in every ascending-member sum, so
+// the sums over the other members are formed once and each level appends
+// x's terms -- the same operations in the same order as ct_group32, hence
+// the same values, in one pass (and one inlined copy) instead of four.
+__device__ __forceinline__ void ct_group32_x4(const Tables &tb, const DevParams &p, uint32_t m, int x, uint32_t lw,
+                                              float *Tg, float *Eg) {
+  const uint32_t rest = m & ~(1u << x);
+  float U = 0.f, B = 0.f, D = 0.f;
+  for (uint32_t mm = rest; mm; mm &= mm - 1) {
+    const int i = __ffs(mm) - 1, r = i * 4 + (int)((lw >> (2 * i)) & 3u);
+    U += tb.u[r];
+    B += tb.bw[r];
+    D += tb.dh[r];
+  }
+  float Ux[4], Bx[4], Dx[4], Tm[4];
+#pragma unroll
+  for (int l = 0; l < 4; l++) {
+    const int rx = x * 4 + l;
+    Ux[l] = U + tb.u[rx];
+    Bx[l] = B + tb.bw[rx];
+    Dx[l] = D + tb.dh[rx];
+    Tm[l] = 0.f;
+  }
+  // the other members, in ascending order: sigma over the others, then + d[i][x, l]
+  for (uint32_t mm = rest; mm; mm &= mm - 1) {
+    const int i = __ffs(mm) - 1, ri = i * 4 + (int)((lw >> (2 * i)) & 3u);
+    float s = 1.f;
+    for (uint32_t m2 = rest & ~(1u << i); m2; m2 &= m2 - 1) {
+      const int j = __ffs(m2) - 1;
+      s += tb.d[ri * p.ds + j * 4 + (int)((lw >> (2 * j)) & 3u)];
+    }
+#pragma unroll
+    for (int l = 0; l < 4; l++) {
+      const float cg = fmaxf(fmaxf(1.f, Ux[l]), Bx[l]);
+      Tm[l] = fmaxf(Tm[l], tb.th[ri] * (s + tb.d[ri * p.ds + x * 4 + l]) * cg);
+    }
+  }
+  // x itself (its sigma sums the others in ascending order; x is the highest member)
+#pragma unroll
+  for (int l = 0; l < 4; l++) {
+    const int rx = x * 4 + l;
+    float s = 1.f;
+    for (uint32_t m2 = rest; m2; m2 &= m2 - 1) {
+      const int j = __ffs(m2) - 1;
+      s += tb.d[rx * p.ds + j * 4 + (int)((lw >> (2 * j)) & 3u)];
+    }
+    const float cg = fmaxf(fmaxf(1.f, Ux[l]), Bx[l]);
+    float T = fmaxf(Tm[l], tb.th[rx] * s * cg);
+    if (p.model & SCHED_MODEL_POWER_CAP) T = fmaxf(T, Dx[l] * p.kcap);  // R28
+    Tg[l] = T;
+    Eg[l] = p.phat * T + Dx[l];
+  }
+}
+
 __device__ __forceinline__ uint32_t ct_set(uint32_t lw, int x, int l) {
   return (lw & ~(3u << (2 * x))) | ((uint32_t)l << (2 * x));
 }
@@ -246,13 +301,9 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
               Ep += Eg;
             }
             float At[4], Ae[4], Bt[4], Be[4], Ct[4], Ce[4];
-#pragma unroll
-            for (int l = 0; l < 4; l++) {
-              const uint32_t ll = ct_set(ct_set(ct_set(lw, x1, l), x2, l), x3, l);
-              ct_group32(tb, p, ma, ll, At[l], Ae[l]);
-              ct_group32(tb, p, mb, ll, Bt[l], Be[l]);
-              ct_group32(tb, p, mc, ll, Ct[l], Ce[l]);
-            }
+            ct_group32_x4(tb, p, ma, x1, lw, At, Ae);
+            ct_group32_x4(tb, p, mb, x2, lw, Bt, Be);
+            ct_group32_x4(tb, p, mc, x3, lw, Ct, Ce);
             if (whole) {
               // the tile's 64 configurations, min-reduced to the exact lower corner
               float mT = __int_as_float(0x7f800000), mE = mT;
@@ -292,14 +343,18 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
               Ep64 = __dadd_rn(Ep64, Eg);
             }
             double A64[4], AE64[4], B64[4], BE64[4], C64[4], CE64[4];
+#pragma unroll 1  // rare path: keep the code small (instruction cache)
             for (int l = 0; l < 4; l++) {
               const uint32_t ll = ct_set(ct_set(ct_set(lw, x1, l), x2, l), x3, l);
               ct_group64(tb, p, ma, ll, A64[l], AE64[l]);
               ct_group64(tb, p, mb, ll, B64[l], BE64[l]);
               ct_group64(tb, p, mc, ll, C64[l], CE64[l]);
             }
+#pragma unroll 1
             for (int a = 0; a < 4; a++)
+#pragma unroll 1
               for (int b = 0; b < 4; b++)
+#pragma unroll 1
                 for (int c = 0; c < 4; c++) {
                   const uint32_t v = vo | ((uint32_t)a << s1) | ((uint32_t)b << s2) | ((uint32_t)c << s3);
                   if (v < v0 || v >= v1) continue;
