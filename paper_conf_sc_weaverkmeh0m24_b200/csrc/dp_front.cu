@@ -204,8 +204,25 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       }
   }
   const double ps = p.ps;
-  double lt = __longlong_as_double(0x7ff0000000000000ll), le = lt;  // the lane's last inserted point
+  const double kInf = __longlong_as_double(0x7ff0000000000000ll);
+  double lt = kInf, le = kInf;  // the lane's last inserted point
+  double bt = kInf, be = kInf;  // the lane's lowest-(T, E) evaluated point
+  // every lane runs the same number of blocks: the warp can share its best point
+  const bool uni = v0 % Lh == 0 && (v1 - v0) % (32ull * Lh) == 0;
   for (uint64_t hv = v0 / Lh + lane; hv * Lh < v1; hv += 32) {
+    double wt = kInf, we = kInf;  // the warp's lowest-(T, E) evaluated point (a real point of B)
+    if (uni) {
+      wt = bt;
+      we = be;
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        const double t2 = __shfl_xor_sync(0xffffffffu, wt, o), e2 = __shfl_xor_sync(0xffffffffu, we, o);
+        if (t2 < wt || (t2 == wt && e2 < we)) {
+          wt = t2;
+          we = e2;
+        }
+      }
+    }
     int rh[kMS - kH];
     double sg[kMS - kH];
     double U = 0.0, Bw = 0.0, D = 0.0;
@@ -257,12 +274,13 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       // a deeper low member is formed once at its loop level -- the same
       // additions in the same ascending-member order as below.
       const int r0b = mw[nh] * L, r1b = mw[nh + 1] * L, r2b = mw[nh + 2] * L;
-      if (nf > 0) {
+      if (nf > 0 || wt != kInf) {
         // Block lower corner: every canonical sum with each low member's term
         // replaced by its minimum over the levels (same order; rounding is
         // monotone, all terms >= 0), so T >= Tmin and E >= Emin for every
-        // vector of the block.  A front point at or below the corner
-        // dominates (or equals) all 64 vectors: skip the block.
+        // vector of the block.  A point of B at or below the corner (the
+        // lane's front, or the warp's best evaluated point) dominates or
+        // equals all 64 vectors: skip the block.
         const int rb[kH] = {r0b, r1b, r2b};
         double Umin = U, Bmin = Bw, Dmin = D;
 #pragma unroll
@@ -318,8 +336,8 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
           if (tcap > Tmin) Tmin = tcap;
         }
         const double Emin = __dadd_rn(__dmul_rn(ps, Tmin), Dmin);
-        bool skip = false;
-        for (int i = 0; i < nf; i++)
+        bool skip = wt <= Tmin && we <= Emin;
+        for (int i = 0; i < nf && !skip; i++)
           if (f[i].t <= Tmin && f[i].e <= Emin) {
             skip = true;
             break;
@@ -377,6 +395,10 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
             x.pad = 0;
             // quick reject: a point inserted earlier (lt, le) dominates or equals x ->
             // so does the front (transitivity), front_insert would keep it unchanged
+            if (x.t < bt || (x.t == bt && x.e < be)) {
+              bt = x.t;
+              be = x.e;
+            }
             if (x.t >= lt && x.e >= le) continue;
             ok &= front_insert<kLF>(f, nf, x);
             lt = x.t;
