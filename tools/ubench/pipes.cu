@@ -12,6 +12,14 @@ __device__ __forceinline__ float max2f(float a, float b) {
   float d; asm volatile("max.f32 %0, %1, %2;" : "=f"(d) : "f"(a), "f"(b)); return d; }
 __device__ __forceinline__ float add1f(float a, float b) {
   float d; asm volatile("add.rn.f32 %0, %1, %2;" : "=f"(d) : "f"(a), "f"(b)); return d; }
+__device__ __forceinline__ unsigned iadd3(unsigned a, unsigned b, unsigned c) {
+  unsigned d; asm volatile("add.u32 %0, %1, %2;\n\tadd.u32 %0, %0, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c)); return d; }
+__device__ __forceinline__ unsigned lop3(unsigned a, unsigned b, unsigned c) {
+  unsigned d; asm volatile("lop3.b32 %0, %1, %2, %3, 0x96;" : "=r"(d) : "r"(a), "r"(b), "r"(c)); return d; }
+__device__ __forceinline__ unsigned imad(unsigned a, unsigned b, unsigned c) {
+  unsigned d; asm volatile("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c)); return d; }
+__device__ __forceinline__ float ffma(float a, float b, float c) {
+  float d; asm volatile("fma.rn.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c)); return d; }
 __device__ __forceinline__ unsigned long long add2f(unsigned long long a, unsigned long long b) {
   unsigned long long d; asm volatile("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b)); return d; }
 
@@ -20,8 +28,12 @@ template <int OP>
 __global__ void k(float *out, long long *clk, float s) {
   float x[8];
   unsigned long long y[8];
-  for (int i = 0; i < 8; i++) { x[i] = s * (threadIdx.x + i); y[i] = __float_as_uint(x[i]) * 0x100000001ull; }
+  unsigned z[8];
+  __shared__ float sh[1024];
+  for (int i = threadIdx.x; i < 1024; i += blockDim.x) sh[i] = s * i;
+  for (int i = 0; i < 8; i++) { x[i] = s * (threadIdx.x + i); y[i] = __float_as_uint(x[i]) * 0x100000001ull; z[i] = threadIdx.x * 7 + i; }
   const float xs = s * 0.5f;
+  const unsigned zs = 0x9e3779b9u;
   const unsigned long long ys = y[7] ^ 0x1ull;
   __syncthreads();
   long long t0 = clock64();
@@ -37,12 +49,16 @@ __global__ void k(float *out, long long *clk, float s) {
       if (OP == 5) { x[i] = max3f(x[i], s, xs); y[i] = add2f(y[i], ys); }
       if (OP == 6) { x[i] = max3f(x[i], s, xs); x[(i + 4) & 7] = add1f(x[(i + 4) & 7], s); }
       if (OP == 7) { x[i] = max2f(x[i], s); y[i] = add2f(y[i], ys); }
+      if (OP == 8) z[i] = lop3(z[i], zs, z[(i + 1) & 7]);
+      if (OP == 9) z[i] = imad(z[i], zs, z[(i + 1) & 7]);
+      if (OP == 10) x[i] = ffma(x[i], s, xs);
+      if (OP == 11) x[i] = x[i] + sh[(z[i] + i * 33 + r) & 1023];
     }
   }
   __syncthreads();
   long long t1 = clock64();
   float a = 0;
-  for (int i = 0; i < 8; i++) a += x[i] + __uint_as_float((unsigned)y[i]);
+  for (int i = 0; i < 8; i++) a += x[i] + __uint_as_float((unsigned)y[i]) + (float)z[i];
   out[blockIdx.x * blockDim.x + threadIdx.x] = a;
   if (threadIdx.x == 0) clk[blockIdx.x] = t1 - t0;
 }
@@ -85,6 +101,10 @@ int main() {
     run<5>("FMNMX3 + FADD2 interleaved", 2, bps);
     run<6>("FMNMX3 + FADD interleaved", 2, bps);
     run<7>("FMNMX + FADD2 interleaved", 2, bps);
+    run<8>("LOP3", 1, bps);
+    run<9>("IMAD", 1, bps);
+    run<10>("FFMA", 1, bps);
+    run<11>("LDS (loads only; +LOP3,IADD,FADD each)", 1, bps);
   }
   return 0;
 }
