@@ -188,9 +188,15 @@ __host__ __device__ inline size_t acc64_bytes(const DevParams &p) {
 }
 constexpr size_t kAcc64Max = 40 << 10;  // staged only if it fits beside 4 CTAs per SM
 
+// per-warp scratch of the block-corner bounds (one group per warp item):
+// MD[(k*4 + level of high member k)*3 + j] = min over the levels of low member
+// j of d[high k][low j]; ML[(j*4 + l)*3 + j2] = min over the levels of j2 of
+// d[low j at l][low j2]; then the minima of u, bw, dyn of each low member
+constexpr int kScrMD = (kMS - kH) * 4 * kH, kScrML = kH * 4 * kH, kScr = kScrMD + kScrML + 3 * kH;
+
 template <class A>
 __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32_t B, int s, uint64_t v0,
-                                         uint64_t v1, int lane, PPt *f, int &nf, bool &ok) {
+                                         uint64_t v1, int lane, PPt *f, int &nf, bool &ok, double *scr) {
   const int L = p.L, nh = s - kH;
   const uint32_t Lh = (uint32_t)(L * L * L);
   int mw[kMS];
@@ -204,6 +210,33 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       }
   }
   const double ps = p.ps;
+  {  // the group's corner-bound tables, once per item, lanes cooperating
+    for (int e = lane; e < kScr; e += 32) {
+      double v = 0.0;
+      if (e < kScrMD) {
+        const int k = e / (4 * kH), lk = (e / kH) % 4, j = e % kH;
+        if (k < nh && lk < L) {
+          const int rk = mw[k] * L + lk, rj = mw[nh + j] * L;
+          v = tb.dd(rk * p.ds + rj);
+          for (int l = 1; l < L; l++) v = fmin(v, tb.dd(rk * p.ds + rj + l));
+        }
+      } else if (e < kScrMD + kScrML) {
+        const int x = e - kScrMD, j = x / (4 * kH), l = (x / kH) % 4, j2 = x % kH;
+        if (l < L && j2 != j) {
+          const int rj = mw[nh + j] * L + l, r2 = mw[nh + j2] * L;
+          v = tb.dd(rj * p.ds + r2);
+          for (int l2 = 1; l2 < L; l2++) v = fmin(v, tb.dd(rj * p.ds + r2 + l2));
+        }
+      } else {
+        const int x = e - kScrMD - kScrML, what = x / kH, j = x % kH, rj = mw[nh + j] * L;
+        v = what == 0 ? tb.uu(rj) : what == 1 ? tb.bb(rj) : tb.dyn(rj);
+        for (int l = 1; l < L; l++)
+          v = fmin(v, what == 0 ? tb.uu(rj + l) : what == 1 ? tb.bb(rj + l) : tb.dyn(rj + l));
+      }
+      scr[e] = v;
+    }
+    __syncwarp();
+  }
   const double kInf = __longlong_as_double(0x7ff0000000000000ll);
   double lt = kInf, le = kInf;  // the lane's last inserted point
   double bt = kInf, be = kInf;  // the lane's lowest-(T, E) evaluated point
@@ -243,29 +276,32 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
         Bw = __dadd_rn(Bw, tb.bb(r));
         D = __dadd_rn(D, tb.dyn(r));
       }
+    // sigma prefixes over the high members (ascending q, one rolled loop
+    // with the member's row recomputed from hv: small code), and for each
+    // low member and level the sum over the high members
+    double Q[kH][4];
 #pragma unroll
-    for (int k = 0; k < kMS - kH; k++)
-      if (k < nh) {
-        double a = 1.0;
-#pragma unroll
-        for (int q = 0; q < kMS - kH; q++)
-          if (q < nh && q != k) a = __dadd_rn(a, tb.dd(rh[k] * p.ds + rh[q]));
-        sg[k] = a;
-      }
-    double Q[kH][4];  // low member j at level l: 1 + sum over the high members
+    for (int k = 0; k < kMS - kH; k++) sg[k] = 1.0;
 #pragma unroll
     for (int j = 0; j < kH; j++)
 #pragma unroll
-      for (int l = 0; l < 4; l++) {
-        double a = 1.0;
-        if (l < L) {
-          const int rj = mw[nh + j] * L + l;
+      for (int l = 0; l < 4; l++) Q[j][l] = 1.0;
+    {
+      uint32_t pw = 1;
+      for (int q = 1; q < nh; q++) pw *= (uint32_t)L;  // L^(nh-1): weight of member 0's digit
+#pragma unroll 1
+      for (int q = 0; q < nh; q++, pw /= (uint32_t)L) {
+        const int rq = mw[q] * L + (int)(((uint32_t)hv / pw) % (uint32_t)L);
 #pragma unroll
-          for (int q = 0; q < kMS - kH; q++)
-            if (q < nh) a = __dadd_rn(a, tb.dd(rj * p.ds + rh[q]));
-        }
-        Q[j][l] = a;
+        for (int k = 0; k < kMS - kH; k++)
+          if (k < nh && k != q) sg[k] = __dadd_rn(sg[k], tb.dd(rh[k] * p.ds + rq));
+#pragma unroll
+        for (int j = 0; j < kH; j++)
+#pragma unroll
+          for (int l = 0; l < 4; l++)
+            if (l < L) Q[j][l] = __dadd_rn(Q[j][l], tb.dd((mw[nh + j] * L + l) * p.ds + rq));
       }
+    }
     const uint64_t base = hv * Lh;
     const uint32_t lv0 = (uint32_t)(v0 > base ? v0 - base : 0), lv1 = (uint32_t)(v1 - base < Lh ? v1 - base : Lh);
     if (lv0 == 0 && lv1 == Lh) {
@@ -282,18 +318,13 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
         // lane's front, or the warp's best evaluated point) dominates or
         // equals all 64 vectors: skip the block.
         const int rb[kH] = {r0b, r1b, r2b};
+        const double *MD = scr, *ML = scr + kScrMD, *MX = scr + kScrMD + kScrML;
         double Umin = U, Bmin = Bw, Dmin = D;
 #pragma unroll
         for (int j = 0; j < kH; j++) {
-          double um = tb.uu(rb[j]), bm = tb.bb(rb[j]), dm = tb.dyn(rb[j]);
-          for (int l = 1; l < L; l++) {
-            um = fmin(um, tb.uu(rb[j] + l));
-            bm = fmin(bm, tb.bb(rb[j] + l));
-            dm = fmin(dm, tb.dyn(rb[j] + l));
-          }
-          Umin = __dadd_rn(Umin, um);
-          Bmin = __dadd_rn(Bmin, bm);
-          Dmin = __dadd_rn(Dmin, dm);
+          Umin = __dadd_rn(Umin, MX[j]);
+          Bmin = __dadd_rn(Bmin, MX[kH + j]);
+          Dmin = __dadd_rn(Dmin, MX[2 * kH + j]);
         }
         if ((p.model & SCHED_MODEL_NO_INTERFERENCE) && (Umin > 1.0 || Bmin > 1.0)) continue;  // all infeasible
         double cmin = 1.0;
@@ -303,13 +334,8 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
 #pragma unroll
         for (int k = 0; k < kMS - kH; k++)
           if (k < nh) {
-            double a = sg[k];
-#pragma unroll
-            for (int j = 0; j < kH; j++) {
-              double dmn = tb.dd(rh[k] * p.ds + rb[j]);
-              for (int l = 1; l < L; l++) dmn = fmin(dmn, tb.dd(rh[k] * p.ds + rb[j] + l));
-              a = __dadd_rn(a, dmn);
-            }
+            const double *md = MD + (k * 4 + (rh[k] - mw[k] * L)) * kH;
+            const double a = __dadd_rn(__dadd_rn(__dadd_rn(sg[k], md[0]), md[1]), md[2]);
             const double ts = __dmul_rn(tb.t(rh[k]), a);
             if (ts > mx) mx = ts;
           }
@@ -320,11 +346,7 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
             double a = Q[j][l];
 #pragma unroll
             for (int j2 = 0; j2 < kH; j2++)
-              if (j2 != j) {
-                double dmn = tb.dd((rb[j] + l) * p.ds + rb[j2]);
-                for (int l2 = 1; l2 < L; l2++) dmn = fmin(dmn, tb.dd((rb[j] + l) * p.ds + rb[j2] + l2));
-                a = __dadd_rn(a, dmn);
-              }
+              if (j2 != j) a = __dadd_rn(a, ML[(j * 4 + l) * kH + j2]);
             const double ts = __dmul_rn(tb.t(rb[j] + l), a);
             tj = l == 0 ? ts : fmin(tj, ts);
           }
@@ -488,6 +510,8 @@ __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams 
     __syncthreads();
   }
   const Acc32 a32{tb, dp.p.ps};
+  double *scr = (double *)(sm + ((dp.p.blob_bytes + 15) & ~15u) + (use64 ? acc64_bytes(dp.p) : 0)) +
+                (size_t)(threadIdx.x >> 5) * kScr;  // this warp's corner-bound tables
   for (;;) {
     unsigned long long it = 0;
     if (lane == 0) it = atomicAdd(dp.ctr + kDpItem, 1ull);
@@ -511,8 +535,8 @@ __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams 
     bool ok = true;
     int lev[kMaxN];
     if (dp.p.scope == SCHED_PER_CLIENT && s > kH && s <= kMS && dp.p.L <= 4) {
-      if (use64) pf_split(a64, dp.p, B, s, v0, v1, lane, f, nf, ok);
-      else pf_split(a32, dp.p, B, s, v0, v1, lane, f, nf, ok);
+      if (use64) pf_split(a64, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
+      else pf_split(a32, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
     } else {
       for (uint64_t v = v0 + lane; v < v1; v += 32) {
         decode_vec(dp.p, B, (uint32_t)v, lev);
@@ -898,7 +922,8 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
   CKD(cudaEventRecord(e0, s));
   int nl = 0;
   const size_t smem = ((p.blob_bytes + 15) & ~15u) +
-                      (p.scope == SCHED_PER_CLIENT && acc64_bytes(p) <= kAcc64Max ? acc64_bytes(p) : 0);
+                      (p.scope == SCHED_PER_CLIENT && acc64_bytes(p) <= kAcc64Max ? acc64_bytes(p) : 0) +
+                      sizeof(double) * kScr * (256 / 32);
   CKD(cudaFuncSetAttribute(k_pf_items, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   if (dp.nfull > 0) {
     k_pf_items<<<nsm * 4, 256, smem, s>>>(dp);
