@@ -487,6 +487,13 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
   }
 }
 
+// the fp32-table path out of line: only for tables too large for the fp64
+// shared-memory copies; keeps the hot kernel's code (instruction cache) small
+__device__ __noinline__ void pf_split_a32(const Acc32 &tb, const DevParams &p, uint32_t B, int s, uint64_t v0,
+                                          uint64_t v1, int lane, PPt *f, int &nf, bool &ok, double *scr) {
+  pf_split(tb, p, B, s, v0, v1, lane, f, nf, ok, scr);
+}
+
 // phase 1a: work item = (group, 2^kItemLog2 level vectors); one warp per item
 __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams dp) {
   extern __shared__ __align__(16) unsigned char sm[];
@@ -536,7 +543,7 @@ __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams 
     int lev[kMaxN];
     if (dp.p.scope == SCHED_PER_CLIENT && s > kH && s <= kMS && dp.p.L <= 4) {
       if (use64) pf_split(a64, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
-      else pf_split(a32, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
+      else pf_split_a32(a32, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
     } else {
       for (uint64_t v = v0 + lane; v < v1; v += 32) {
         decode_vec(dp.p, B, (uint32_t)v, lev);
