@@ -494,6 +494,21 @@ __device__ __noinline__ void pf_split_a32(const Acc32 &tb, const DevParams &p, u
   pf_split(tb, p, B, s, v0, v1, lane, f, nf, ok, scr);
 }
 
+// small groups and PER_GPU: one from-scratch fp64 evaluation per level
+// vector (out of line: small code in the hot kernel)
+__device__ __noinline__ void pf_plain(const Tables &tb, const DevParams &p, uint32_t B, uint64_t v0, uint64_t v1,
+                                      int lane, PPt *f, int &nf, bool &ok) {
+  int lev[kMaxN];
+  for (uint64_t v = v0 + lane; v < v1; v += 32) {
+    decode_vec(p, B, (uint32_t)v, lev);
+    PPt x;
+    if (!group64(tb, p, B, lev, x.t, x.e)) continue;
+    x.v = (uint32_t)v;
+    x.pad = 0;
+    ok &= front_insert<kLF>(f, nf, x);
+  }
+}
+
 // phase 1a: work item = (group, 2^kItemLog2 level vectors); one warp per item
 __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams dp) {
   extern __shared__ __align__(16) unsigned char sm[];
@@ -540,19 +555,11 @@ __global__ void __launch_bounds__(256, SCHED_PF_MINB) k_pf_items(const DpParams 
     PPt f[kLF];
     int nf = 0;
     bool ok = true;
-    int lev[kMaxN];
     if (dp.p.scope == SCHED_PER_CLIENT && s > kH && s <= kMS && dp.p.L <= 4) {
       if (use64) pf_split(a64, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
       else pf_split_a32(a32, dp.p, B, s, v0, v1, lane, f, nf, ok, scr);
     } else {
-      for (uint64_t v = v0 + lane; v < v1; v += 32) {
-        decode_vec(dp.p, B, (uint32_t)v, lev);
-        PPt x;
-        if (!group64(tb, dp.p, B, lev, x.t, x.e)) continue;
-        x.v = (uint32_t)v;
-        x.pad = 0;
-        ok &= front_insert<kLF>(f, nf, x);
-      }
+      pf_plain(tb, dp.p, B, v0, v1, lane, f, nf, ok);
     }
     if (!ok) atomicExch(dp.ctr + kDpErr, 1ull);
     // warp merge: every lane keeps its points not dominated by another lane's
