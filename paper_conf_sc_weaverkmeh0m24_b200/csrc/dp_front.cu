@@ -664,27 +664,24 @@ __global__ void __launch_bounds__(256) k_dp_level(const DpParams dp, int m, int 
   DPt f[kFM];
   int nf = 0;
   bool ok = true;
-  const uint32_t nsub = 1u << m;
-  for (uint32_t x = 1 + lane; x < nsub; x += 32) {
-    uint32_t B = 0, xx = x;  // x-th subset of S (bit deposit)
-    for (uint32_t mm = S; mm && xx; mm &= mm - 1, xx >>= 1)
-      if (xx & 1u) B |= mm & (0u - mm);
-    if (!(B & below) || __popc(B) > C) continue;
+  // one candidate last group B of S: B meets `below`, |B| <= C, PF(B) non-empty
+  auto visit = [&](uint32_t B) {
+    if (!(B & below) || __popc(B) > C) return;
     const int sb = dp.sid[B];
-    if (sb < 0) continue;
+    if (sb < 0) return;
     const int npf = dp.pfcnt[sb];
-    if (!npf) continue;
+    if (!npf) return;
     const uint32_t R = S & ~B;
     if (R == 0) {
-      if (k != 1) continue;
+      if (k != 1) return;
       for (int q = 0; q < npf; q++) {
         const PPt b = dp.pf[(size_t)sb * kOF + q];
         DPt y{b.t, b.e, B, 0xff, (uint8_t)q, 0};
         ok &= front_insert<kFM>(f, nf, y);
       }
-      continue;
+      return;
     }
-    if (k == 1 || !(R & 1u)) continue;
+    if (k == 1 || !(R & 1u)) return;
     const size_t src = ((size_t)(R >> 1) * (G + 1) + (k - 1));
     const int nr = dp.frcnt[src];
     for (int i = 0; i < nr; i++) {
@@ -693,6 +690,62 @@ __global__ void __launch_bounds__(256) k_dp_level(const DpParams dp, int m, int 
         const PPt b = dp.pf[(size_t)sb * kOF + q];
         DPt y{a.t > b.t ? a.t : b.t, __dadd_rn(a.e, b.e), B, (uint8_t)i, (uint8_t)q, 0};
         ok &= front_insert<kFM>(f, nf, y);
+      }
+    }
+  };
+  if (C <= 4 && C < m) {
+    // capped groups: enumerate the <= C-subsets of S directly (O(m^C) instead
+    // of all 2^m subsets), lanes split by the subset's lowest member
+    int mem[32];
+    int nm = 0;
+    for (uint32_t mm = S; mm; mm &= mm - 1) mem[nm++] = __ffs(mm) - 1;
+    for (int i1 = lane; i1 < nm; i1 += 32) {
+      const uint32_t b1 = 1u << mem[i1];
+      visit(b1);
+      if (C < 2) continue;
+      for (int i2 = i1 + 1; i2 < nm; i2++) {
+        const uint32_t b2 = b1 | (1u << mem[i2]);
+        visit(b2);
+        if (C < 3) continue;
+        for (int i3 = i2 + 1; i3 < nm; i3++) {
+          const uint32_t b3 = b2 | (1u << mem[i3]);
+          visit(b3);
+          if (C < 4) continue;
+          for (int i4 = i3 + 1; i4 < nm; i4++) visit(b3 | (1u << mem[i4]));
+        }
+      }
+    }
+  } else {
+    const uint32_t nsub = 1u << m;
+    for (uint32_t x = 1 + lane; x < nsub; x += 32) {
+      uint32_t B = 0, xx = x;  // x-th subset of S (bit deposit)
+      for (uint32_t mm = S; mm && xx; mm &= mm - 1, xx >>= 1)
+        if (xx & 1u) B |= mm & (0u - mm);
+      if (!(B & below) || __popc(B) > C) continue;
+      const int sb = dp.sid[B];
+      if (sb < 0) continue;
+      const int npf = dp.pfcnt[sb];
+      if (!npf) continue;
+      const uint32_t R = S & ~B;
+      if (R == 0) {
+        if (k != 1) continue;
+        for (int q = 0; q < npf; q++) {
+          const PPt b = dp.pf[(size_t)sb * kOF + q];
+          DPt y{b.t, b.e, B, 0xff, (uint8_t)q, 0};
+          ok &= front_insert<kFM>(f, nf, y);
+        }
+        continue;
+      }
+      if (k == 1 || !(R & 1u)) continue;
+      const size_t src = ((size_t)(R >> 1) * (G + 1) + (k - 1));
+      const int nr = dp.frcnt[src];
+      for (int i = 0; i < nr; i++) {
+        const DPt a = dp.fr[src * kFM + i];
+        for (int q = 0; q < npf; q++) {
+          const PPt b = dp.pf[(size_t)sb * kOF + q];
+          DPt y{a.t > b.t ? a.t : b.t, __dadd_rn(a.e, b.e), B, (uint8_t)i, (uint8_t)q, 0};
+          ok &= front_insert<kFM>(f, nf, y);
+        }
       }
     }
   }
