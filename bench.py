@@ -166,6 +166,17 @@ def run_reference(args):
     return 0
 
 
+def describe(name, q):
+    """The workload's one-line description (BASELINE.json configs, synth/configs.py)."""
+    idx = {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}.get(name)
+    w = ",".join("[" + "x".join(["T"] * a + ["E"] * b) + "]" for a, b in q.weights)
+    lv = "{" + ",".join(str(x) for x in q.levels) + "}%"
+    return (f"{name}: {q.n} workflows x {q.g} GPUs, <= {q.c} clients per GPU, MPS levels {lv} "
+            f"{'PER_GPU' if q.scope == 1 else 'PER_CLIENT'}, objectives {w}"
+            f"{' + Pareto' if q.want_pareto else ''}"
+            + (f" (BASELINE configs[{idx}])" if idx is not None else ""))
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -300,9 +311,8 @@ def run_ours(args):
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": f"{args.workload}: 16 workflows x 8 GPUs x 4 MPS levels {{25,50,75,100}}%, "
-                               "PER_GPU levels, objectives [TxE],[TxTxE] + Pareto (BASELINE configs[3]); "
-                               f"step = 1/{SLICES} cyclic chunk slice of the space split over ranks",
+        "config": {"workload": describe(args.workload, q) +
+                               f"; step = 1/{SLICES} cyclic chunk slice of the space split over ranks",
                    "space_configs": space, "slices": SLICES, "chunk_log2": CHUNK_LOG2,
                    "time_to_optimal_schedule_s_extrapolated": SLICES * ms_per_step / 1e3,
                    "time_to_optimal_schedule_subset_dp": dp,

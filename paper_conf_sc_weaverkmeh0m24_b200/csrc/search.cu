@@ -622,7 +622,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   }
   DevParams dp_full = dp;
   const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
-                    (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 26);  // >= 2^38 configs
+                    (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 20);  // >= 2^32 configs
   for (int pass = seed ? 0 : 1; pass < 3; pass++) {
     dp = dp_full;
     if (pass == 0) {
