@@ -35,7 +35,7 @@ def space(n, g, c, L, scope):
     return out
 
 
-COUNT_IDLE, NO_INTERFERENCE, POWER_CAP = 1, 2, 4   # scoring-model variants (R26-R28)
+COUNT_IDLE, NO_INTERFERENCE, POWER_CAP, TIME_SLICE = 1, 2, 4, 8   # scoring-model variants (R26-R28, R30)
 
 
 def _capped(t, dyn, capd):
@@ -97,17 +97,26 @@ def score(prof, n, rgs, lv_prof, model=0, pcap=0.0, g=1):
             return False, None, None
         cg = max(max(1.0, U), B)
         Tg = 0.0
-        for i in grp:
-            s = 1.0
-            for j in grp:
-                if j != i:
-                    s = s + d[i, lv_prof[i], j, lv_prof[j]]
-            tau = (t[i, lv_prof[i]] * s) * cg
-            Tg = max(Tg, tau)
+        if model & TIME_SLICE:
+            # R30: no MPS, the members take turns on the
+            # whole GPU at their solo profile; each slice capped on its own
+            for i in grp:
+                ti = t[i, lv_prof[i]]
+                if model & POWER_CAP:
+                    ti = _capped(ti, (p[i, lv_prof[i]] - ps) * ti, float(pcap) - ps)
+                Tg = Tg + ti
+        else:
+            for i in grp:
+                s = 1.0
+                for j in grp:
+                    if j != i:
+                        s = s + d[i, lv_prof[i], j, lv_prof[j]]
+                tau = (t[i, lv_prof[i]] * s) * cg
+                Tg = max(Tg, tau)
         D = 0.0
         for i in grp:
             D = D + (p[i, lv_prof[i]] - ps) * t[i, lv_prof[i]]
-        if model & POWER_CAP:
+        if model & POWER_CAP and not model & TIME_SLICE:
             Tg = _capped(Tg, D, float(pcap) - ps)
         T = max(T, Tg)
         E = E + (ps * Tg + D)

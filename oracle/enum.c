@@ -37,7 +37,7 @@
  *  Pareto set of distinct (T,E) over feasible configurations, one (lowest)
  *  index per point.
  *
- *  Scoring-model variants (readings R26-R28 in DESIGN.md),
+ *  Scoring-model variants (readings R26-R28, R30 in DESIGN.md),
  *  selected by or_query.model bits; 0 is the canonical model above:
  *   1 COUNT_IDLE: every one of the G GPUs draws P_s for the whole makespan
  *     (R8 variant).  With E_g = P_s*T_g + D_g this is
@@ -55,6 +55,16 @@
  *     A solo task in the sequential baseline likewise runs for
  *     t' = max(t, dyn / (P_cap - P_s)); its energy stays p*t when not capped,
  *     else P_s*t' + dyn.
+ *   8 TIME_SLICE: time slicing instead of MPS (without
+ *     MPS the clients of a GPU take turns on the whole device; reading R30):
+ *     nothing runs concurrently, so there is no contention stretch c_g and
+ *     no co-run slowdown; each member runs its own slice at its solo
+ *     profile, one after another:
+ *       T_g = sum_{i in g, ascending} tau_i,  tau_i = t_i,
+ *     with POWER_CAP each slice is throttled on its own like a solo task of
+ *     the sequential baseline: tau_i = max(t_i, dyn_i / (P_cap - P_s));
+ *       E_g = P_s*T_g + D_g.
+ *     (Not combined with NO_INTERFERENCE, a rule about concurrent clients.)
  */
 #include <stdint.h>
 #include <stdlib.h>
@@ -79,7 +89,7 @@ typedef struct {
   const int *wa, *wb;      /* [nw] exponents */
   uint64_t lo, hi;         /* index window [lo, hi) */
   int want_pareto;
-  unsigned model;          /* variant bits: 1 COUNT_IDLE, 2 NO_INTERFERENCE, 4 POWER_CAP */
+  unsigned model;          /* variant bits: 1 COUNT_IDLE, 2 NO_INTERFERENCE, 4 POWER_CAP, 8 TIME_SLICE */
   float power_cap;         /* P_cap (W) for POWER_CAP */
   double tseq_base, eseq_base;  /* > 0: sequential baselines given by the caller (the unsplit
                                    queue of a split search, R29); 0: computed below */
@@ -88,6 +98,7 @@ typedef struct {
 #define OR_COUNT_IDLE 1u
 #define OR_NO_INTERFERENCE 2u
 #define OR_POWER_CAP 4u
+#define OR_TIME_SLICE 8u
 
 typedef struct { uint64_t idx; double f, t, e; int found; } or_best;
 typedef struct { uint64_t idx; double t, e; } or_point;
@@ -230,19 +241,30 @@ int oracle_score_config(const or_profile *P, const or_query *q, int n, const int
     if (U > c) c = U;
     if (B > c) c = B;
     double Tg = 0.0;
-    for (int i = 0; i < n; i++) if (a[i] == g) {
-      double sigma = 1.0;
-      for (int j = 0; j < n; j++) if (a[j] == g && j != i)
-        sigma = sigma + (double)P->d[((size_t)(i * lp + pl[i]) * P->n + j) * lp + pl[j]];
-      double tau = ((double)P->t[i * lp + pl[i]] * sigma) * c;
-      if (tau > Tg) Tg = tau;
+    if (q->model & OR_TIME_SLICE) {          /* R30: the slices one after another */
+      for (int i = 0; i < n; i++) if (a[i] == g) {
+        double tau = (double)P->t[i * lp + pl[i]];
+        if (q->model & OR_POWER_CAP) {
+          double tc = (((double)P->p[i * lp + pl[i]] - ps) * (double)P->t[i * lp + pl[i]]) / capd;
+          if (tc > tau) tau = tc;
+        }
+        Tg = Tg + tau;
+      }
+    } else {
+      for (int i = 0; i < n; i++) if (a[i] == g) {
+        double sigma = 1.0;
+        for (int j = 0; j < n; j++) if (a[j] == g && j != i)
+          sigma = sigma + (double)P->d[((size_t)(i * lp + pl[i]) * P->n + j) * lp + pl[j]];
+        double tau = ((double)P->t[i * lp + pl[i]] * sigma) * c;
+        if (tau > Tg) Tg = tau;
+      }
     }
     double D = 0.0;
     for (int i = 0; i < n; i++) if (a[i] == g) {
       double dyn = ((double)P->p[i * lp + pl[i]] - ps) * (double)P->t[i * lp + pl[i]];
       D = D + dyn;
     }
-    if (q->model & OR_POWER_CAP) {
+    if ((q->model & OR_POWER_CAP) && !(q->model & OR_TIME_SLICE)) {
       double tc = D / capd;
       if (tc > Tg) Tg = tc;
     }

@@ -23,7 +23,7 @@ class Query:
     index_lo: int = 0
     index_hi: int | None = None   # None = |Omega|
     model: int = 0                # scoring-model variant bits (R26-R28): 1 COUNT_IDLE,
-    power_cap: float = 0.0        # 2 NO_INTERFERENCE, 4 POWER_CAP (P_cap in W)
+    power_cap: float = 0.0        # 2 NO_INTERFERENCE, 4 POWER_CAP (P_cap in W), 8 TIME_SLICE (R30)
     tseq_base: float = 0.0        # > 0: sequential baselines supplied by the caller (the
     eseq_base: float = 0.0        # unsplit queue of a split search, R29)
 
