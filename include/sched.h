@@ -61,7 +61,7 @@ enum {
 enum { SCHED_PER_CLIENT = 0, SCHED_PER_GPU = 1 };
 
 /* Scoring-model variants (sched_query.model_flags; readings
- * R26-R28 in DESIGN.md).  0 = the canonical model.
+ * R26-R28, R30 in DESIGN.md).  0 = the canonical model.
  *  COUNT_IDLE       every one of the g GPUs draws the static power P_s for
  *                   the whole makespan: E = g*P_s*T + sum_g D_g, and the
  *                   sequential baseline E_seq = g*P_s*T_seq + sum_i dyn_i (R8 variant).
@@ -72,8 +72,24 @@ enum { SCHED_PER_CLIENT = 0, SCHED_PER_GPU = 1 };
  *                   300 W on A100X): a group is throttled until its average
  *                   power is <= P_cap with its dynamic energy conserved,
  *                   T_g' = max(T_g, D_g / (P_cap - P_s)); solo tasks of the
- *                   sequential baseline likewise. */
-enum { SCHED_MODEL_COUNT_IDLE = 1, SCHED_MODEL_NO_INTERFERENCE = 2, SCHED_MODEL_POWER_CAP = 4 };
+ *                   sequential baseline likewise.
+ *  TIME_SLICE       time slicing instead of MPS (the
+ *                   default CUDA sharing, processes take turns on the whole
+ *                   GPU; reading R30): no concurrent execution, so no
+ *                   contention stretch and no co-run slowdown; the clients
+ *                   of a group run one after another at their solo profile,
+ *                   T_g = sum_i tau_i (members ascending), tau_i = t_i, or
+ *                   under POWER_CAP tau_i = max(t_i, dyn_i/(P_cap - P_s))
+ *                   (each slice throttled on its own, as the sequential
+ *                   baseline); E_g = P_s*T_g + D_g.  Cannot be combined with
+ *                   NO_INTERFERENCE (a concurrency rule): SCHED_E_INVALID.
+ *                   Searched by the generic kernel; sched_front_dp rejects it. */
+enum {
+  SCHED_MODEL_COUNT_IDLE = 1,
+  SCHED_MODEL_NO_INTERFERENCE = 2,
+  SCHED_MODEL_POWER_CAP = 4,
+  SCHED_MODEL_TIME_SLICE = 8
+};
 
 #define SCHED_MAX_WORKFLOWS 32
 #define SCHED_MAX_GPUS 16
@@ -223,7 +239,8 @@ int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int
  * vectors, then the block-order DP over workflow subsets.  Reaches spaces
  * that cannot be enumerated, e.g. the literal per-client c4 (16 workflows,
  * 8 GPUs, 4 levels per client: 4.05e19 configurations).  Requires
- * 2 <= n <= 20, L^max_clients <= 2^32 (PER_CLIENT), no SCHED_MODEL_COUNT_IDLE;
+ * 2 <= n <= 20, L^max_clients <= 2^32 (PER_CLIENT), no SCHED_MODEL_COUNT_IDLE
+ * or SCHED_MODEL_TIME_SLICE;
  * the index window and shard fields must be the defaults (whole space, one
  * shard).  front[front_cap] is ordered by X descending (T ascending), one
  * witness configuration per distinct (T, E); best[W] is the max F_w over the

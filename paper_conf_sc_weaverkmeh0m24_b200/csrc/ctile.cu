@@ -11,7 +11,7 @@ static size_t ctile_smem(const DevParams &dp) {
 
 bool ctile_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.scope != SCHED_PER_CLIENT || dp.L != 4 || dp.n < 6 || dp.n > 15) return false;
-  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE)) return false;
+  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE | SCHED_MODEL_TIME_SLICE)) return false;
   tl->fn = dp.nw <= 1 ? ctile_fn<1>() : dp.nw <= 2 ? ctile_fn<2>() : dp.nw <= 4 ? ctile_fn<4>() : ctile_fn<8>();
   tl->smem = ctile_smem(dp);
   return true;

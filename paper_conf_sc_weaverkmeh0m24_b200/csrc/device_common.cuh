@@ -201,7 +201,18 @@ __device__ __forceinline__ void refine64(const Tables &tb, const DevParams &p, c
     if (U > c) c = U;
     if (B > c) c = B;
     double Tg = 0.0;
-    for (uint32_t mm = m; mm; mm &= mm - 1) {
+    if (p.model & SCHED_MODEL_TIME_SLICE) {  // R30: slices one after another at the solo profile
+      for (uint32_t mm = m; mm; mm &= mm - 1) {
+        const int r = (__ffs(mm) - 1) * p.L + lam[__ffs(mm) - 1];
+        double tau = (double)tb.traw[r];
+        if (p.model & SCHED_MODEL_POWER_CAP) {
+          const double tc = __ddiv_rn(__dmul_rn(__dsub_rn((double)tb.praw[r], ps), tau), p.capd);
+          if (tc > tau) tau = tc;
+        }
+        Tg = __dadd_rn(Tg, tau);
+      }
+    }
+    for (uint32_t mm = (p.model & SCHED_MODEL_TIME_SLICE) ? 0u : m; mm; mm &= mm - 1) {
       const int i = __ffs(mm) - 1, ri = i * p.L + lam[i];
       double sigma = 1.0;
       for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) {
@@ -216,7 +227,7 @@ __device__ __forceinline__ void refine64(const Tables &tb, const DevParams &p, c
       const int i = __ffs(mm) - 1, r = i * p.L + lam[i];
       D = __dadd_rn(D, __dmul_rn(__dsub_rn((double)tb.praw[r], ps), (double)tb.traw[r]));
     }
-    if (p.model & SCHED_MODEL_POWER_CAP) {  // R28
+    if ((p.model & (SCHED_MODEL_POWER_CAP | SCHED_MODEL_TIME_SLICE)) == SCHED_MODEL_POWER_CAP) {  // R28
       const double tc = __ddiv_rn(D, p.capd);
       if (tc > Tg) Tg = tc;
     }

@@ -918,7 +918,8 @@ void dp_groups(const Profile &P, const Query &q, std::vector<uint32_t> *smask, s
 }  // namespace
 
 int dp_front_workspace(const Profile &P, const Query &q, const DevParams &dp, size_t *bytes) {
-  if (q.n < 2 || q.n > 20 || q.g > kMaxG || (q.model & SCHED_MODEL_COUNT_IDLE)) return SCHED_E_INVALID;
+  if (q.n < 2 || q.n > 20 || q.g > kMaxG || (q.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_TIME_SLICE)))
+    return SCHED_E_INVALID;
   if (q.scope == SCHED_PER_CLIENT) {
     double lg = 0.0;  // L^C must fit the 32-bit vector id
     for (int k = 0; k < q.c; k++) lg += std::log2((double)q.L);

@@ -97,8 +97,11 @@ int resolve_query_shape(const sched_query *q, int n_profile_levels, Query *Q) {
   Q->cand_cap = q->candidate_cap == 0 ? (1u << 20) : q->candidate_cap;
   Q->lo = q->index_lo;
   Q->hi = q->index_hi;
-  if (q->model_flags & ~(uint32_t)(SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE | SCHED_MODEL_POWER_CAP))
+  if (q->model_flags & ~(uint32_t)(SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE | SCHED_MODEL_POWER_CAP |
+                                    SCHED_MODEL_TIME_SLICE))
     return SCHED_E_INVALID;
+  if ((q->model_flags & SCHED_MODEL_TIME_SLICE) && (q->model_flags & SCHED_MODEL_NO_INTERFERENCE))
+    return SCHED_E_INVALID;  // R30: the hard rule is about concurrent clients
   Q->model = q->model_flags;
   Q->pcap = q->power_cap_w;
   if ((Q->model & SCHED_MODEL_POWER_CAP) && !(std::isfinite(Q->pcap) && Q->pcap > 0.f)) return SCHED_E_INVALID;
@@ -459,7 +462,19 @@ int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const i
     if (U > c) c = U;
     if (B > c) c = B;
     double Tg = 0.0;
-    for (int i = 0; i < n; i++) {
+    if (q.model & SCHED_MODEL_TIME_SLICE) {  // R30: slices one after another, solo profile
+      for (int i = 0; i < n; i++) {
+        if (a[i] != g) continue;
+        const size_t r = (size_t)i * lp + pl[i];
+        double tau = (double)P.t[r];
+        if (q.model & SCHED_MODEL_POWER_CAP) {
+          const double tc = (((double)P.p[r] - ps) * (double)P.t[r]) / ((double)q.pcap - ps);
+          if (tc > tau) tau = tc;
+        }
+        Tg = Tg + tau;
+      }
+    }
+    for (int i = 0; i < n && !(q.model & SCHED_MODEL_TIME_SLICE); i++) {
       if (a[i] != g) continue;
       double sigma = 1.0;
       for (int j = 0; j < n; j++)
@@ -474,7 +489,7 @@ int host_score(const Profile &P, const Query &q, const int8_t *a, int k, const i
         const size_t r = (size_t)i * lp + pl[i];
         D = D + ((double)P.p[r] - ps) * (double)P.t[r];
       }
-    if (q.model & SCHED_MODEL_POWER_CAP) {  // R28
+    if ((q.model & SCHED_MODEL_POWER_CAP) && !(q.model & SCHED_MODEL_TIME_SLICE)) {  // R28
       const double tc = D / ((double)q.pcap - ps);
       if (tc > Tg) Tg = tc;
     }
@@ -630,7 +645,10 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->n_units = dp->n_owned << (dp->chunk_log2 - dp->unit_log2);
   dp->unit_stride = 1;
   dp->cand_cap = q.cand_cap;
-  dp->gtab_ok = ((uint64_t)L << n) * sizeof(GroupRec) <= ((uint64_t)384 << 20);
+  // R30 (TIME_SLICE) is scored by the generic kernel only: no group table, so
+  // the tile / suffix / DFS paths are not eligible.
+  dp->gtab_ok = ((uint64_t)L << n) * sizeof(GroupRec) <= ((uint64_t)384 << 20) &&
+                !(dp->model & SCHED_MODEL_TIME_SLICE);
   {  // interleave lanes when partitions hold enough level vectors to keep lanes together
     double per = 1.0;
     const int nd = q.scope == SCHED_PER_CLIENT ? n : std::min(q.g, n);

@@ -85,13 +85,20 @@ __device__ __forceinline__ void score32_inc(const Tables &tb, const DevParams &p
     }
     const float cg = fmaxf(fmaxf(1.f, U), B);
     float Tg = 0.f;
-    for (uint32_t mm = m; mm; mm &= mm - 1) {
-      const int i = __ffs(mm) - 1, ri = i * p.L + lam[i];
-      float s = 1.f;
-      for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) s += tb.d[ri * p.ds + (__ffs(m2) - 1) * p.L + lam[__ffs(m2) - 1]];
-      Tg = fmaxf(Tg, tb.th[ri] * s * cg);
+    if (p.model & SCHED_MODEL_TIME_SLICE) {  // R30: sum of the solo slices (per-slice cap)
+      for (uint32_t mm = m; mm; mm &= mm - 1) {
+        const int r = (__ffs(mm) - 1) * p.L + lam[__ffs(mm) - 1];
+        Tg += (p.model & SCHED_MODEL_POWER_CAP) ? fmaxf(tb.th[r], tb.dh[r] * p.kcap) : tb.th[r];
+      }
+    } else {
+      for (uint32_t mm = m; mm; mm &= mm - 1) {
+        const int i = __ffs(mm) - 1, ri = i * p.L + lam[i];
+        float s = 1.f;
+        for (uint32_t m2 = m & ~(1u << i); m2; m2 &= m2 - 1) s += tb.d[ri * p.ds + (__ffs(m2) - 1) * p.L + lam[__ffs(m2) - 1]];
+        Tg = fmaxf(Tg, tb.th[ri] * s * cg);
+      }
+      if (p.model & SCHED_MODEL_POWER_CAP) Tg = fmaxf(Tg, D * p.kcap);  // R28
     }
-    if (p.model & SCHED_MODEL_POWER_CAP) Tg = fmaxf(Tg, D * p.kcap);  // R28
     gc.t[g] = Tg;
     gc.e[g] = p.phat * Tg + D;
     gc.d[g] = D;

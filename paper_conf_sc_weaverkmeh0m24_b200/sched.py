@@ -25,9 +25,10 @@ SCHED_E_WORKSPACE = -6
 SCHED_E_NODEVICE = -7
 PER_CLIENT = 0
 PER_GPU = 1
-SCHED_MODEL_COUNT_IDLE = 1        # scoring-model variants (include/sched.h, R26-R28)
+SCHED_MODEL_COUNT_IDLE = 1        # scoring-model variants (include/sched.h, R26-R28, R30)
 SCHED_MODEL_NO_INTERFERENCE = 2
 SCHED_MODEL_POWER_CAP = 4
+SCHED_MODEL_TIME_SLICE = 8       # R30: time slicing instead of MPS (generic kernel)
 UINT64_MAX = (1 << 64) - 1
 
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",

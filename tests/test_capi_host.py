@@ -89,11 +89,11 @@ def test_host_score_bitwise_oracle(name):
                 assert p.score64 == oracle.objective(ts, es, T, E, a, b)
 
 
-@pytest.mark.parametrize("model", [1, 2, 4, 7])
+@pytest.mark.parametrize("model", [1, 2, 4, 7, 8, 9, 12, 13])
 @pytest.mark.parametrize("name", ["c2", "c4", "c5"])
 def test_host_score_variants_bitwise_oracle(name, model):
     """Library fp64 host score (sched_score) under the scoring-model variants
-    (R26-R28) == the oracle's, bitwise, including the variant baselines."""
+    (R26-R28, R30) == the oracle's, bitwise, including the variant baselines."""
     import dataclasses
     prof, q = config(name)
     q = dataclasses.replace(q, model=model, power_cap=180.0)
@@ -115,11 +115,13 @@ def test_host_score_variants_bitwise_oracle(name, model):
 
 
 def test_variant_queries_validated():
-    """POWER_CAP needs P_cap > P_s; unknown model bits are rejected."""
+    """POWER_CAP needs P_cap > P_s; unknown model bits and TIME_SLICE with
+    NO_INTERFERENCE (R30) are rejected."""
     import dataclasses
     prof, q = config("c1")
     sch = S.Scheduler(prof)
-    for bad in (dict(model=4, power_cap=50.0), dict(model=4, power_cap=0.0), dict(model=8)):
+    for bad in (dict(model=4, power_cap=50.0), dict(model=4, power_cap=0.0), dict(model=16),
+                dict(model=10)):
         with pytest.raises(S.SchedError) as e:
             sch.score(dataclasses.replace(q, **bad), 0, 0)
         assert e.value.status == S.sched.SCHED_E_INVALID

@@ -1,5 +1,6 @@
 """GPU parity of the scoring-model variants (include/sched.h SCHED_MODEL_*,
-DESIGN.md R26 COUNT_IDLE, R27 NO_INTERFERENCE, R28 POWER_CAP) on every
+DESIGN.md R26 COUNT_IDLE, R27 NO_INTERFERENCE, R28 POWER_CAP, R30
+TIME_SLICE) on every
 kernel path that accepts them, against the oracle (same bar as
 test_gpu_parity.check: bitwise picks, Pareto set and counts)."""
 import dataclasses
@@ -15,7 +16,7 @@ from test_gpu_parity import check
 pytestmark = pytest.mark.gpu
 
 W = ((1, 0), (0, 1), (1, 1), (2, 1))
-MODELS = [1, 2, 4, 3, 5, 6, 7]
+MODELS = [1, 2, 4, 3, 5, 6, 7, 8, 9, 12, 13]
 
 
 @pytest.mark.parametrize("model", MODELS)
@@ -62,7 +63,7 @@ def test_power_cap_tile_kernel(monkeypatch):
     check(res, oracle.search(prof, q), q)
 
 
-@pytest.mark.parametrize("name,model", [("c4", 4), ("c5", 6), ("c3", 1), ("c2", 2)])
+@pytest.mark.parametrize("name,model", [("c4", 4), ("c5", 6), ("c3", 1), ("c2", 2), ("c4", 8), ("c2", 12)])
 def test_variants_big_windows(name, model):
     """Windows of the BASELINE workloads under a variant (P_cap = 300 W, the
     paper's A100X cap), in the default launch configuration."""
