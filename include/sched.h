@@ -83,7 +83,9 @@ enum { SCHED_PER_CLIENT = 0, SCHED_PER_GPU = 1 };
  *                   (each slice throttled on its own, as the sequential
  *                   baseline); E_g = P_s*T_g + D_g.  Cannot be combined with
  *                   NO_INTERFERENCE (a concurrency rule): SCHED_E_INVALID.
- *                   Searched by the generic kernel; sched_front_dp rejects it. */
+ *                   Scored through the group table (tile / suffix / pair
+ *                   kernels) or the generic kernel; the PER_CLIENT tile
+ *                   kernel declines it and sched_front_dp rejects it. */
 enum {
   SCHED_MODEL_COUNT_IDLE = 1,
   SCHED_MODEL_NO_INTERFERENCE = 2,

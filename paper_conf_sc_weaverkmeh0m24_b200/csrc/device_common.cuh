@@ -423,7 +423,21 @@ __device__ __forceinline__ bool group_eval(const Tables &tb, const DevParams &p,
   if (B64 > c) c = B64;
   float Tg = 0.f;
   double Tg64 = 0.0;
-  for (uint32_t mm = m; mm; mm &= mm - 1) {
+  if (p.model & SCHED_MODEL_TIME_SLICE) {  // R30: the slices one after another (per-slice cap)
+    for (uint32_t mm = m; mm; mm &= mm - 1) {
+      const int r = (__ffs(mm) - 1) * L + mu;
+      double tau = (double)tb.traw[r];
+      if (p.model & SCHED_MODEL_POWER_CAP) {
+        Tg += fmaxf(tb.th[r], tb.dh[r] * p.kcap);
+        const double tc = __ddiv_rn(__dmul_rn(__dsub_rn((double)tb.praw[r], p.ps), tau), p.capd);
+        if (tc > tau) tau = tc;
+      } else {
+        Tg += tb.th[r];
+      }
+      Tg64 = __dadd_rn(Tg64, tau);
+    }
+  }
+  for (uint32_t mm = (p.model & SCHED_MODEL_TIME_SLICE) ? 0u : m; mm; mm &= mm - 1) {
     const int i = __ffs(mm) - 1, ri = i * L + mu;
     float s = 1.f;
     double s64 = 1.0;
@@ -440,7 +454,8 @@ __device__ __forceinline__ bool group_eval(const Tables &tb, const DevParams &p,
     const int r = (__ffs(mm) - 1) * L + mu;
     D64 = __dadd_rn(D64, __dmul_rn(__dsub_rn((double)tb.praw[r], p.ps), (double)tb.traw[r]));
   }
-  if (p.model & SCHED_MODEL_POWER_CAP) {  // R28: throttled to P_cap, dynamic energy conserved
+  if ((p.model & (SCHED_MODEL_POWER_CAP | SCHED_MODEL_TIME_SLICE)) == SCHED_MODEL_POWER_CAP) {
+    // R28: throttled to P_cap, dynamic energy conserved
     Tg = fmaxf(Tg, D * p.kcap);
     const double tc = __ddiv_rn(D64, p.capd);
     if (tc > Tg64) Tg64 = tc;

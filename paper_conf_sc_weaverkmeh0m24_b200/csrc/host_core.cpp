@@ -645,10 +645,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->n_units = dp->n_owned << (dp->chunk_log2 - dp->unit_log2);
   dp->unit_stride = 1;
   dp->cand_cap = q.cand_cap;
-  // R30 (TIME_SLICE) is scored by the generic kernel only: no group table, so
-  // the tile / suffix / DFS paths are not eligible.
-  dp->gtab_ok = ((uint64_t)L << n) * sizeof(GroupRec) <= ((uint64_t)384 << 20) &&
-                !(dp->model & SCHED_MODEL_TIME_SLICE);
+  dp->gtab_ok = ((uint64_t)L << n) * sizeof(GroupRec) <= ((uint64_t)384 << 20);
   {  // interleave lanes when partitions hold enough level vectors to keep lanes together
     double per = 1.0;
     const int nd = q.scope == SCHED_PER_CLIENT ? n : std::min(q.g, n);

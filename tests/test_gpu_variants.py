@@ -39,11 +39,11 @@ def test_variants_small_generic_and_auto(model, seed, monkeypatch):
     check(res, ref, q)
 
 
-@pytest.mark.parametrize("model", [2, 4, 6])
+@pytest.mark.parametrize("model", [2, 4, 6, 8, 12])
 @pytest.mark.parametrize("kernel,path", [("sfx", 3), ("dfs", 2)])
 def test_variants_partition_kernels(model, kernel, path, monkeypatch):
-    """L = 1: NO_INTERFERENCE / POWER_CAP enter through the group table on
-    the suffix and pair kernels."""
+    """L = 1: NO_INTERFERENCE / POWER_CAP / TIME_SLICE enter through the
+    group table on the suffix and pair kernels."""
     monkeypatch.setenv("SCHED_KERNEL", kernel)
     prof = make_profile(10, levels=(100,), seed=41, g=5, c=3)
     sweep = ((1, 0), (3, 1), (2, 1), (1, 1), (1, 2), (1, 3), (0, 1))   # a weight set the pair kernel is built for
@@ -53,17 +53,19 @@ def test_variants_partition_kernels(model, kernel, path, monkeypatch):
     check(res, oracle.search(prof, q), q)
 
 
-def test_power_cap_tile_kernel(monkeypatch):
-    """POWER_CAP on the PER_GPU L = 4 tile kernel (group-local)."""
+@pytest.mark.parametrize("model", [4, 8, 12])
+def test_power_cap_tile_kernel(model, monkeypatch):
+    """POWER_CAP / TIME_SLICE on the PER_GPU L = 4 tile kernel (group-local,
+    through the group table)."""
     monkeypatch.setenv("SCHED_KERNEL", "tile")
     prof = make_profile(9, levels=(25, 50, 75, 100), seed=42)
-    q = Query(9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 1), (2, 1)), True, model=4, power_cap=130.0)
+    q = Query(9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 1), (2, 1)), True, model=model, power_cap=130.0)
     res = S.Scheduler(prof).search(q)
     assert res.stats["kernel_path"] == 1
     check(res, oracle.search(prof, q), q)
 
 
-@pytest.mark.parametrize("name,model", [("c4", 4), ("c5", 6), ("c3", 1), ("c2", 2), ("c4", 8), ("c2", 12)])
+@pytest.mark.parametrize("name,model", [("c4", 4), ("c5", 6), ("c3", 1), ("c2", 2), ("c4", 8), ("c2", 12), ("c5", 8), ("c3", 12)])
 def test_variants_big_windows(name, model):
     """Windows of the BASELINE workloads under a variant (P_cap = 300 W, the
     paper's A100X cap), in the default launch configuration."""
