@@ -122,3 +122,55 @@ def test_dp_front_c5_equals_certificate():
     for p in list(front) + list(best):
         assert _witness_ok(prof, q, p)
     print("c5 DP:", st["total_ms"], "ms")
+
+
+def _canon(lab):
+    m = {}
+    return [m.setdefault(x, len(m)) for x in lab]
+
+
+def test_dp_front_c4_literal_per_client_no_better_neighbour_or_sample():
+    """Literal per-client c4 (n = 16: no full oracle, DESIGN.md 'parity
+    partial') -- properties every correct front has at any size, checked with
+    the oracle's fp64 scorer: no configuration one move away from a witness
+    (one client's level changed, or one client moved to another / a new
+    group) and none of 20000 seeded random configurations strictly dominates
+    a front point or beats a per-weight optimum.  Catches a DP that drops a
+    level combination, a group split or a subset state."""
+    import random
+    prof, q = config("c4")
+    qc = dataclasses.replace(q, scope=PER_CLIENT)
+    rc, best, front, st = S.Scheduler(prof).front_dp(qc)
+    assert rc == S.sched.SCHED_OK and len(front) > 0
+    pts = [(p.makespan_s, p.energy_j) for p in front]
+    ts, es = oracle.constants(prof, qc)
+    n, L, G = qc.n, len(qc.levels), qc.g
+
+    def check(rgs, digits):
+        ok, T, E = oracle.score(prof, qc, rgs, digits)
+        if not ok:
+            return 0
+        for (pt, pe) in pts:
+            assert not (T <= pt and E <= pe and (T < pt or E < pe)), (rgs, digits, T, E, pt, pe)
+        for w, (a, b) in enumerate(qc.weights):
+            assert oracle.objective(ts, es, T, E, a, b) <= best[w].score64
+        return 1
+
+    nfeas = 0
+    for p in list(front) + list(best):
+        rgs = [int(p.group_of[i]) for i in range(n)]
+        lv = [int(p.level_of[i]) for i in range(n)]
+        k = max(rgs) + 1
+        for i in range(n):
+            for d in range(L):
+                if d != lv[i]:
+                    nfeas += check(rgs, lv[:i] + [d] + lv[i + 1:])
+            for gnew in range(min(k + 1, G)):
+                if gnew != rgs[i]:
+                    lab = rgs[:i] + [gnew] + rgs[i + 1:]
+                    nfeas += check(_canon(lab), lv)
+    rnd = random.Random(16)
+    for _ in range(20000):
+        lab = [rnd.randrange(G) for _ in range(n)]
+        nfeas += check(_canon(lab), [rnd.randrange(L) for _ in range(n)])
+    assert nfeas > 10000
