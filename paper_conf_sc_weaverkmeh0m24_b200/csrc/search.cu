@@ -707,7 +707,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     }
     launches++;
     if (dp.nw > 0) {
-      k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid);
+      k_best_final<<<dp.nw, 256, 0, st>>>(dp, grid * (path == 3 ? tl.slots_per_cta : 1));
       CK(cudaGetLastError());
       launches++;
     }

@@ -474,7 +474,6 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
   Stair stair = stair_at(after);
   SfxWarp<M> *wps = (SfxWarp<M> *)(after + kStairSmem);
   SfxWarp<M> &w = wps[warp];
-  BestRec *red = (BestRec *)(wps + kSfxWarps);
   stair_init(stair);
   if (lane < kSfxMaxG) w.key[lane] = 0xffffffffu;
   for (int i = p.g * RS + lane; i < kSfxMaxG * RS; i += 32)  // rows >= G: no group
@@ -633,22 +632,14 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
     atomicAdd(p.ctr + kCtrFeasible, nfeas);
     atomicAdd(p.ctr + kCtrRefined, nref64);
   }
+  // per-warp best slots (slot = CTA * kSfxWarps + warp; k_best_final reduces
+  // them): no block barrier after the warps' independent unit loops
 #pragma unroll
   for (int q = 0; q < kMaxW; q++) {
     if (q < p.nw) {
       warp_best(cold.lb[q]);
-      if (lane == 0) red[warp * kMaxW + q] = cold.lb[q];
+      if (lane == 0) ((BestRec *)p.slots)[((size_t)blockIdx.x * kSfxWarps + warp) * p.nw + q] = cold.lb[q];
     }
-  }
-  __syncthreads();
-  if (threadIdx.x < p.nw) {
-    const int q = threadIdx.x;
-    BestRec b = red[q];
-    for (int kk = 1; kk < kSfxWarps; kk++) {
-      const BestRec xx = red[kk * kMaxW + q];
-      if (xx.valid && (!b.valid || better(xx.f, xx.idx, b.f, b.idx))) b = xx;
-    }
-    ((BestRec *)p.slots)[(size_t)blockIdx.x * p.nw + q] = b;
   }
 }
 

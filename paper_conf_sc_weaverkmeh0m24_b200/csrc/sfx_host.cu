@@ -18,6 +18,7 @@ bool sfx_eligible(DevParams &dp, TileLaunch *tl) {
   else return false;
   tl->fn = M == 6 ? sfx_fn<6>() : sfx_fn<4>();
   tl->smem = sfx_smem(dp, M);
+  tl->slots_per_cta = kSfxWarps;
   return true;
 }
 
@@ -29,7 +30,7 @@ cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kSfxThreads, tl.smem);
   if (err != cudaSuccess) return err;
   if (occ < 1) return cudaErrorInvalidConfiguration;
-  *grid = std::min(4096, nsm * occ);
+  *grid = std::min(4096 / kSfxWarps, nsm * occ);  // per-warp best slots: grid * kSfxWarps <= kMaxGrid
   if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kSfxWarps;

@@ -23,6 +23,7 @@ const void *tile_fn();
 struct TileLaunch {
   const void *fn;
   size_t smem;
+  int slots_per_cta = 1;  // best slots written per CTA (k_sfx: one per warp)
 };
 
 #ifndef SCHED_TILE_THREADS
