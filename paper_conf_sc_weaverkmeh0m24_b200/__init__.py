@@ -8,3 +8,4 @@ the exact Pareto set.  C ABI: include/sched.h; kernels: csrc/.
 """
 from .sched import (Scheduler, SearchResult, SchedError, Pick, count, unrank, rank, merge,  # noqa: F401
                     version, lib, PER_CLIENT, PER_GPU, EXPORTS)
+from .resume import search_resumable, CoverageError  # noqa: F401,E402
