@@ -20,7 +20,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 CFLAGS = [*ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-ffp-contract=off,-fno-fast-math",
-          "-Xptxas", "-v", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
+          "-Xptxas", "-v", "-Xcompiler", "-iquote," + os.path.join(ROOT, "include"), "-I", CSRC,
+          # include/sched.h only as "sched.h" (-iquote): <sched.h> of the system headers (pthread) stays glibc's
           *os.environ.get("SCHED_NVCC_EXTRA", "").split()]
 
 

@@ -1,6 +1,7 @@
 // capi.cpp -- the extern "C" boundary declared in include/sched.h.
 // Argument checking, handle/cache management, staging, result conversion.
 // No exception crosses the ABI (every entry point catches).
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges for nsys / ncu --nvtx (SURVEY 5 tracing)
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -9,6 +10,14 @@
 #include <new>
 
 #include "sched_internal.hpp"
+
+
+namespace {
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 using namespace sched;
 
@@ -149,6 +158,7 @@ extern "C" {
 
 int sched_create(const sched_profile *profile, sched_handle **out) {
   GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_create");
   if (!out) return SCHED_E_INVALID;
   *out = nullptr;
   sched_handle *h = new sched_handle();
@@ -224,6 +234,7 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
                  sched_pick *best, sched_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto,
                  sched_stats *stats) {
   GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_search");
   if (!h || !ws) return SCHED_E_INVALID;
   int st = need_device();
   if (st) return st;
@@ -311,6 +322,7 @@ int sched_merge(int32_t n_ranks, int32_t n_weights, const sched_pick *rank_best,
                 const sched_pick *rank_pareto, const uint64_t *rank_npareto, sched_pick *best,
                 sched_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto) {
   GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_merge");
   return merge_picks(n_ranks, n_weights, rank_best, rank_pareto, rank_npareto, best, pareto, pareto_cap,
                      n_pareto);
   GUARD_END
@@ -407,6 +419,7 @@ int sched_front_dp(sched_handle *h, const sched_query *qin, void *ws, size_t ws_
                    sched_dp_point *best, sched_dp_point *front, uint64_t front_cap, uint64_t *n_front,
                    sched_stats *stats) {
   GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_front_dp");
   if (!h || !ws || !n_front || (front_cap > 0 && !front)) return SCHED_E_INVALID;
   int st = need_device();
   if (st) return st;
@@ -570,6 +583,7 @@ int sched_search_splits(sched_handle *h, const sched_query *qin, const int32_t *
                         sched_split_pick *pareto, uint64_t pareto_cap, uint64_t *n_pareto,
                         sched_stats *stats) {
   GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_search_splits");
   if (!ws) return SCHED_E_INVALID;
   int st = need_device();
   if (st) return st;
