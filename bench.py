@@ -29,7 +29,7 @@ sys.path.insert(0, ROOT)
 METRIC = "configurations scored/sec (whole box) at 1/2/4/8 B200; time-to-optimal-schedule"
 UNIT = "configs/s"
 SLICES = 64
-CHUNK_LOG2 = 22
+CHUNK_LOG2 = 24   # 2^24-index chunks: tools/chunk_sweep.py (c4 step 669.8 -> 653.0 ms vs 2^22)
 OPS_PER_CONFIG = 4   # T max, E add, 2 min-reductions (c4 tile kernel, per configuration)
 SMS = 148
 LANES_PER_SM_CLK = 4 * 32   # 4 SMSPs x 32 lanes issue slots per clock

@@ -299,7 +299,7 @@ def test_client_tile_kernel_path(n, g, c, ws, pareto, model, seed):
 
 def test_bench_slice_launch_configuration():
     """One bench.py step exactly as it is timed (c4, shard (sigma, 64) of
-    2^22-index chunks, 3.2e12 configurations): coverage equals the slice's
+    2^24-index chunks (bench.CHUNK_LOG2), 3.2e12 configurations): coverage equals the slice's
     index count, every returned configuration re-scores bitwise in the
     oracle, the slice's optimum never beats the O3 certificate's, and no
     sampled oracle window of the slice beats the slice's best or escapes its
@@ -307,7 +307,8 @@ def test_bench_slice_launch_configuration():
     import json
     import os
     prof, q = config("c4")
-    sigma, slices, cl = 5, 64, 22
+    import bench
+    sigma, slices, cl = 5, 64, bench.CHUNK_LOG2
     tot = S.count(q)
     sch = S.Scheduler(prof)
     res = sch.search(q, shard=(sigma, slices), chunk_log2=cl)
