@@ -133,7 +133,7 @@ typedef struct {
   uint64_t index_lo, index_hi;  /* searched window [lo, hi); hi = UINT64_MAX means |Omega| */
   int32_t shard_rank;           /* this rank's share: chunks c with c % shard_count == rank */
   int32_t shard_count;          /* >= 1 (multi-GPU split, one process per GPU) */
-  int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 12..40 (0 = default 22) */
+  int32_t chunk_log2;           /* chunk = 2^chunk_log2 consecutive indices, 12..40 (0 = default 24) */
   int32_t want_pareto;          /* nonzero: also compute the (T, E) Pareto set */
   uint32_t candidate_cap;       /* device Pareto-candidate buffer records; 0 = 1<<20 */
   uint32_t model_flags;         /* SCHED_MODEL_* bits; 0 = canonical model */

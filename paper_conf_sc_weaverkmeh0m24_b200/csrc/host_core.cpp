@@ -91,7 +91,7 @@ int resolve_query_shape(const sched_query *q, int n_profile_levels, Query *Q) {
   Q->count = q->shard_count;
   Q->rank = q->shard_rank;
   if (Q->count < 1 || Q->rank < 0 || Q->rank >= Q->count) return SCHED_E_INVALID;
-  Q->chunk_log2 = q->chunk_log2 == 0 ? 22 : q->chunk_log2;
+  Q->chunk_log2 = q->chunk_log2 == 0 ? 24 : q->chunk_log2;  // 2^24: profiles/r01_chunk_sweep.txt
   if (Q->chunk_log2 < 12 || Q->chunk_log2 > 40) return SCHED_E_INVALID;
   Q->want_pareto = q->want_pareto != 0;
   Q->cand_cap = q->candidate_cap == 0 ? (1u << 20) : q->candidate_cap;

@@ -35,7 +35,8 @@ cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kSfxWarps;
     int ul = 12;
-    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 8) ul++;
+    // <= 2^22: the suffix kernel loses to the last-unit tail with larger units (c5: 752 vs 770 ms at 2^24)
+    while (ul < std::min(dp.chunk_log2, 22) && (range >> (ul + 1)) >= warps * 8) ul++;
     dp.unit_log2 = ul;
     dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
     dp.unit_stride = 1;

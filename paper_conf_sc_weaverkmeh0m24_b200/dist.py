@@ -61,7 +61,7 @@ def exchange(best, pareto, n_weights, group=None, device=None, pareto_cap=1 << 1
     return mb, mp, int(allr.numel() + cnts.numel() * 8)
 
 
-def sharded_search(sched, q, group=None, chunk_log2=22, slices=(0, 1), **kw):
+def sharded_search(sched, q, group=None, chunk_log2=24, slices=(0, 1), **kw):
     """This rank's share of q (optionally one of `slices[1]` cyclic slices of
     the chunk sequence), then exchange + exact merge.  Returns
     (best, pareto, local SearchResult, n_configs summed over ranks)."""

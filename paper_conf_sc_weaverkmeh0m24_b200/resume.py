@@ -61,7 +61,7 @@ def fingerprint(profile, q) -> str:
     return h.hexdigest()
 
 
-def windows_of(total: int, n_windows: int, align: int = 1 << 22):
+def windows_of(total: int, n_windows: int, align: int = 1 << 24):
     """[lo, hi) windows tiling [0, total), boundaries on multiples of `align`
     (the chunk size) where the space allows."""
     n_windows = max(1, n_windows)
@@ -102,12 +102,12 @@ def check_coverage(records, total: int) -> None:
 
 
 def search_resumable(sched, profile, q, path: str, n_windows: int = 64, max_windows: int | None = None,
-                     search_fn=None, pareto_cap: int = 1 << 16, align: int = 1 << 22):
+                     search_fn=None, pareto_cap: int = 1 << 16, align: int = 1 << 24):
     """Exhaustive search of the whole space of `q`, checkpointed per window.
 
     sched: a Scheduler for `profile`.  search_fn(qw) -> SearchResult-like
     (best, pareto, stats["n_configs"]); default sched.search.  align: window
-    boundaries on multiples of this (default the 2^22 chunk).  max_windows:
+    boundaries on multiples of this (default the 2^24 chunk).  max_windows:
     stop after searching that many NEW windows (simulates an interrupted
     run); returns None then.  Otherwise returns (best[W], pareto, stats)
     with stats = {"n_configs", "n_feasible", "windows", "resumed"}.

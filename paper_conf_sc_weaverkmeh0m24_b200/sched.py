@@ -174,7 +174,7 @@ class Scheduler:
             pass
 
     # -- query marshalling --
-    def cquery(self, q, shard=(0, 1), chunk_log2=22, candidate_cap=0):
+    def cquery(self, q, shard=(0, 1), chunk_log2=24, candidate_cap=0):
         mask = 0
         for v in q.levels:
             mask |= 1 << self.level_pct.index(int(v))

@@ -94,7 +94,7 @@ def test_windows_big_spaces(name):
     tot = S.count(q)
     sch = S.Scheduler(prof)
     rnd = random.Random(11)
-    for lo, hi in _windows(tot, 1 << 22, rnd, 300_000):
+    for lo, hi in _windows(tot, 1 << 24, rnd, 300_000):
         qw = q.with_range(lo, hi)
         check(sch.search(qw), oracle.search(prof, qw), qw)
 

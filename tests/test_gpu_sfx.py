@@ -87,7 +87,7 @@ def test_sfx_c5_windows(sfx):
     tot = S.count(q)
     sch = S.Scheduler(prof)
     rnd = random.Random(17)
-    wins = [(0, 200_000), (tot - 200_000, tot), ((1 << 22) - 100_000, (1 << 22) + 100_000)]
+    wins = [(0, 200_000), (tot - 200_000, tot), ((1 << 24) - 100_000, (1 << 24) + 100_000)]
     wins += [(x, x + 200_000) for x in (rnd.randrange(tot - 200_000) for _ in range(4))]
     for lo, hi in wins:
         qw = q.with_range(lo, hi)

@@ -117,8 +117,8 @@ def test_gpu_resumed_search_equals_one_shot(tmp_path):
     q = Query(9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 1), (2, 1)), True)
     sch = S.Scheduler(prof)
     ck = str(tmp_path / "ck.jsonl")
-    assert R.search_resumable(sch, prof, q, ck, n_windows=7, max_windows=2) is None
-    best, par, st = R.search_resumable(sch, prof, q, ck, n_windows=7)
+    assert R.search_resumable(sch, prof, q, ck, n_windows=7, max_windows=2, align=1 << 20) is None
+    best, par, st = R.search_resumable(sch, prof, q, ck, n_windows=7, align=1 << 20)
     one = sch.search(q)
     assert st["resumed"] == 2 and st["n_configs"] == one.stats["n_configs"]
     assert [b.index for b in best] == one.best_indices and [b.score64 for b in best] == [b.score64 for b in one.best]
