@@ -245,17 +245,81 @@ def objective(tseq, eseq, T, E, a, b) -> float:
     return lib().oracle_objective(tseq, eseq, T, E, a, b)
 
 
-def dp_certificate(prof, q, cap: int = 1 << 20):
+def _client_fronts(args):
+    """Phase 1 of O4 for groups B in [b_lo, b_hi): (off[b_hi - b_lo + 1], t, e)."""
+    prof, q, b_lo, b_hi = args[:4]
+    batched = args[4] if len(args) > 4 else 1
+    pk = _Pack(prof, q)
+    lev = (C.c_int * len(pk.lev_idx))(*pk.lev_idx)
+    f = lib().oracle_client_fronts
+    f.restype = C.c_longlong
+    off = np.zeros(b_hi - b_lo + 1, np.int64)
+    cap = 1 << 16
+    while True:
+        t = np.zeros(cap, np.float64)
+        e = np.zeros(cap, np.float64)
+        n = f(C.byref(pk.P), q.n, min(q.c, q.n), len(q.levels), lev, C.c_uint(b_lo), C.c_uint(b_hi),
+              _ptr(t, C.c_double), _ptr(e, C.c_double), _ptr(off, C.c_longlong), C.c_longlong(cap),
+              int(batched))
+        if n >= 0:
+            return off, t[:n].copy(), e[:n].copy()
+        cap *= 4
+
+
+def _client_tasks(n, c, L, parts):
+    """Split [1, 2^n) into ~parts ranges of similar cost (L^|B| |B|^2 per group)."""
+    cost = [0.0] * (1 << n)
+    for B in range(1, 1 << n):
+        s = bin(B).count("1")
+        cost[B] = float(L) ** s * (s * s + 4) if s <= c else 0.0
+    tot = sum(cost)
+    out, lo, acc = [], 0, 0.0
+    for B in range(1 << n):
+        acc += cost[B]
+        if acc >= tot / parts or B == (1 << n) - 1:
+            out.append((lo, B + 1))
+            lo, acc = B + 1, 0.0
+    return out
+
+
+def client_fronts_parallel(prof, q, procs: int, parts: int | None = None):
+    """Phase 1 of O4 over a process pool; returns (off[2^n + 1], t, e)."""
+    tasks = _client_tasks(q.n, min(q.c, q.n), len(q.levels), parts or procs * 16)
+    # largest tasks first so the pool's tail is short
+    order = sorted(range(len(tasks)), key=lambda i: tasks[i][0] - tasks[i][1])
+    res = [None] * len(tasks)
+    with ProcessPoolExecutor(procs) as ex:
+        futs = {i: ex.submit(_client_fronts, (prof, q, *tasks[i])) for i in order}
+        for i in order:
+            res[i] = futs[i].result()
+    offs, ts, es, base = [], [], [], 0
+    for off, t, e in res:
+        offs.append(off[:-1] + base)
+        ts.append(t)
+        es.append(e)
+        base += t.size
+    off = np.concatenate(offs + [np.array([base], np.int64)])
+    return off, np.concatenate(ts), np.concatenate(es)
+
+
+def dp_certificate(prof, q, cap: int = 1 << 20, procs: int = 1):
     """O3 (PER_GPU) / O4 (PER_CLIENT) in dpcert.c: exact Pareto-front values
     [(T, E)] (T ascending) of the whole space and the exact optimum F per
-    weight (max over the front, canonical fp64).  Values only, no indices."""
+    weight (max over the front, canonical fp64).  Values only, no indices.
+    procs > 1 (PER_CLIENT): O4's per-group fronts in a process pool over
+    disjoint group ranges, then the same DP (oracle_client_dp)."""
     assert getattr(q, "model", 0) == 0, "certificate covers the canonical model"
     pk = _Pack(prof, q)
     ot = (C.c_double * cap)()
     oe = (C.c_double * cap)()
     lev = (C.c_int * len(pk.lev_idx))(*pk.lev_idx)
-    fn = lib().oracle_dpcert if q.scope == 1 else lib().oracle_dpcert_client   # O3 / O4
-    nf = fn(C.byref(pk.P), q.n, q.g, min(q.c, q.n), len(q.levels), lev, ot, oe, cap)
+    if q.scope == 0 and procs > 1:
+        off, t, e = client_fronts_parallel(prof, q, procs)
+        nf = lib().oracle_client_dp(q.n, q.g, _ptr(t, C.c_double), _ptr(e, C.c_double),
+                                    _ptr(off, C.c_longlong), ot, oe, cap)
+    else:
+        fn = lib().oracle_dpcert if q.scope == 1 else lib().oracle_dpcert_client   # O3 / O4
+        nf = fn(C.byref(pk.P), q.n, q.g, min(q.c, q.n), len(q.levels), lev, ot, oe, cap)
     if nf < 0:
         raise RuntimeError("certificate capacity / size")
     front = [(ot[i], oe[i]) for i in range(nf)]

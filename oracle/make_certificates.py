@@ -3,11 +3,13 @@
 
   python -m oracle.make_certificates            # c3, c4, c5 (O3)
   python -m oracle.make_certificates client 14  # O4: the first 14 workflows of c4, per-client levels
+  python -m oracle.make_certificates client 16 7  # O4 at the full c4 (n = 16), phase 1 on 7 processes
 """
 import dataclasses
 import json
 import os
 import sys
+import time
 
 import oracle
 from synth import config
@@ -29,16 +31,19 @@ def main():
         print(name, len(c["front"]), c["best"])
 
 
-def client(n: int):
+def client(n: int, procs: int = 1):
     """O4 (PER_CLIENT) certificate of the c4 profile's first n workflows with
     c4's G = 8, 4 levels, uncapped clients: the literal per-client reading
     at the largest size O4 can run (n = 14: 5^14 level-vector groups)."""
     prof, q = config("c4")
     q = dataclasses.replace(q, n=n, scope=0, weights=((1, 1), (2, 1), (1, 0), (0, 1)))
-    c = oracle.dp_certificate(prof.subset(n), q)
+    t0 = time.time()
+    c = oracle.dp_certificate(prof.subset(n), q, procs=procs)
+    wall = time.time() - t0
     out = {"config": f"c4 first {n} workflows, PER_CLIENT", "n": n, "g": q.g, "c": q.c,
            "levels": list(q.levels), "scope": "PER_CLIENT",
            "source": "oracle.dp_certificate (oracle/dpcert.c, O4), seed 0 synth.config('c4').subset(n)",
+           "oracle_procs": procs, "oracle_wall_s": round(wall, 1),
            "weights": [list(w) for w in q.weights],
            "tseq": c["tseq"].hex(), "eseq": c["eseq"].hex(),
            "best_score64": [b.hex() for b in c["best"]],
@@ -50,6 +55,6 @@ def client(n: int):
 
 if __name__ == "__main__":
     if len(sys.argv) > 2 and sys.argv[1] == "client":
-        client(int(sys.argv[2]))
+        client(int(sys.argv[2]), int(sys.argv[3]) if len(sys.argv) > 3 else 1)
     else:
         main()

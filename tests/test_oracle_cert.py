@@ -62,3 +62,33 @@ def test_client_certificate_equals_enumeration(n, g, c, levels, seed):
     cert = oracle.dp_certificate(prof, q)
     assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
     assert [b[1] if b else None for b in r["best"]] == cert["best"]
+
+
+@pytest.mark.parametrize("n,c,levels,seed", [
+    (7, 7, (25, 50, 75, 100), 710), (8, 4, (50, 100), 711), (6, 6, (25, 75, 100), 712), (9, 3, (100,), 713),
+])
+def test_client_fronts_batched_equals_plain(n, c, levels, seed):
+    """O4 phase 1: the batched per-group fronts (last member's levels swept
+    inside group_tuples_last, prefix sums shared) equal the plain form
+    (every level vector through group_tuple_members) bitwise for every group,
+    including groups made infeasible by memory (WarpX / BerkeleyGW rows)."""
+    from synth import PER_CLIENT
+    arch = [11, 2, 0, 12, 5, 1, 7, 9, 3][:n]
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed, archetypes=arch)
+    q = Query(n, n, c, levels, PER_CLIENT, W, True)
+    off0, t0, e0 = oracle._client_fronts((prof, q, 0, 1 << n, 0))
+    off1, t1, e1 = oracle._client_fronts((prof, q, 0, 1 << n, 1))
+    assert off0.tolist() == off1.tolist()
+    assert t0.tobytes() == t1.tobytes() and e0.tobytes() == e1.tobytes()
+    assert (off0[1:] == off0[:-1]).any()   # some group infeasible (memory)
+
+
+def test_client_certificate_parallel_equals_serial():
+    """The process-pool form of O4 (phase 1 split over group ranges) equals
+    the one-process O4 bitwise."""
+    from synth import PER_CLIENT
+    prof = make_profile(9, levels=(25, 50, 75, 100), seed=720)
+    q = Query(9, 4, 9, (50, 100), PER_CLIENT, W, True)
+    a = oracle.dp_certificate(prof, q)
+    b = oracle.dp_certificate(prof, q, procs=3)
+    assert a["front"] == b["front"] and a["best"] == b["best"]
