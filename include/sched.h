@@ -230,6 +230,20 @@ int sched_unrank(const sched_query *q, uint64_t index, int8_t *group_of, int8_t 
 int sched_rank(const sched_query *q, const int8_t *group_of, const int8_t *level_of,
                uint64_t *index);
 
+/* Device unrank (SURVEY 8(a) H3/H4, 4.2 "device unrank == host unrank"):
+ * for t in [0, n): configuration of index d_index[t] + advance, computed on
+ * the device by the search kernels' own routines -- unrank of d_index[t]
+ * through the DP count table staged in shared memory, then `advance` steps of
+ * the successor walk (level digits, then the next RGS) -- written as
+ * d_group_of[t*q->n + i] / d_level_of[t*q->n + i] (layout of sched_unrank).
+ * Indices (after advance) >= |Omega| give d_group_of[t*q->n] = -1.
+ * d_index, d_group_of, d_level_of are DEVICE pointers owned by the caller;
+ * ws is the query's search workspace (sched_workspace_size); asynchronous on
+ * `stream` (no host sync).  SCHED_E_INVALID on a bad query or null pointer. */
+int sched_unrank_device(sched_handle *h, const sched_query *q, const uint64_t *d_index, uint64_t n,
+                        uint64_t advance, int8_t *d_group_of, int8_t *d_level_of, void *ws,
+                        size_t ws_bytes, void *stream);
+
 /* fp64 canonical score of one configuration on the host, weight w (0..W-1;
  * with W == 0 score64 = X).  out->valid = 0 if memory-infeasible.  Host only. */
 int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int32_t w,

@@ -9,6 +9,7 @@
 #include <cstring>
 #include <new>
 
+#include "event_guard.hpp"
 #include "sched_internal.hpp"
 
 
@@ -249,8 +250,9 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
   st = build_stage(h->P, q, *sp, &blob, &dp);
   if (st) return st;
   if (ws_bytes < workspace_bytes(dp, 0) || ((uintptr_t)ws & 255)) return SCHED_E_WORKSPACE;
-  cudaEvent_t t0, t1;
-  if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess) return SCHED_E_CUDA;
+  EventGuard<2> ev;  // destroyed on every return path
+  if (!ev.create()) return SCHED_E_CUDA;
+  cudaEvent_t t0 = ev[0], t1 = ev[1];
   cudaEventRecord(t0, (cudaStream_t)stream);
   uint64_t h2d = 0;
   if (h->staged_ws != ws || h->staged_blob != blob) {
@@ -267,8 +269,6 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
   cudaEventSynchronize(t1);
   float total_ms = 0.f;
   cudaEventElapsedTime(&total_ms, t0, t1);
-  cudaEventDestroy(t0);
-  cudaEventDestroy(t1);
   if (st && st != SCHED_E_CAPACITY) return st;
   if (ctr[kCtrOverflow]) st = SCHED_E_CAPACITY;
   for (int w = 0; w < q.nw; w++) fill_pick(q, dp, w, bres[w], &best[w]);
@@ -357,7 +357,11 @@ int sched_rank(const sched_query *qin, const int8_t *group_of, const int8_t *lev
   if (st) return st;
   int8_t dig[kMaxN];
   int k = 0;
-  for (int i = 0; i < q.n; i++) k = group_of[i] + 1 > k ? group_of[i] + 1 : k;
+  for (int i = 0; i < q.n; i++) {  // validate before any dig[] write (group ids index dig)
+    if (group_of[i] < 0 || group_of[i] >= q.g || group_of[i] >= kMaxG) return SCHED_E_INVALID;
+    if (level_of[i] < 0 || level_of[i] >= q.L) return SCHED_E_INVALID;
+    k = group_of[i] + 1 > k ? group_of[i] + 1 : k;
+  }
   if (q.scope == SCHED_PER_CLIENT) {
     for (int i = 0; i < q.n; i++) dig[i] = level_of[i];
   } else {
@@ -370,6 +374,31 @@ int sched_rank(const sched_query *qin, const int8_t *group_of, const int8_t *lev
     }
   }
   return host_rank(sp, group_of, dig, index);
+  GUARD_END
+}
+
+int sched_unrank_device(sched_handle *h, const sched_query *qin, const uint64_t *d_index, uint64_t n,
+                        uint64_t advance, int8_t *d_group_of, int8_t *d_level_of, void *ws, size_t ws_bytes,
+                        void *stream) {
+  GUARD_BEGIN
+  NvtxRange nvtx_range_("sched_unrank_device");
+  if (!h || !ws || (n > 0 && (!d_index || !d_group_of || !d_level_of))) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  Query q;
+  const Space *sp;
+  st = resolve(h, qin, &q, &sp);
+  if (st) return st;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = build_stage(h->P, q, *sp, &blob, &dp);
+  if (st) return st;
+  if (ws_bytes < workspace_bytes(dp, 0) || ((uintptr_t)ws & 255)) return SCHED_E_WORKSPACE;
+  if (h->staged_ws != ws || h->staged_blob != blob) {
+    st = do_stage(h, dp, blob, ws, stream);
+    if (st) return st;
+  }
+  return launch_unrank(dp, ws, ws_bytes, stream, d_index, n, advance, d_group_of, d_level_of);
   GUARD_END
 }
 

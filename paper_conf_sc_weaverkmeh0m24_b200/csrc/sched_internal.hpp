@@ -194,6 +194,8 @@ struct LaunchInfo {
 size_t workspace_bytes(const DevParams &dp, int max_grid);
 int stage_tables(const DevParams &dp, const std::vector<unsigned char> &blob, void *d_ws, void *host_pinned,
                  void *stream);
+int launch_unrank(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, const uint64_t *d_idx, uint64_t n,
+                  uint64_t advance, int8_t *gout, int8_t *lout);
 int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, LaunchInfo *info,
                   std::vector<BestRec> *best, std::vector<CandRec> *pareto, uint64_t *ctr_out);
 

@@ -20,6 +20,7 @@
 #include <cstring>
 
 #include "device_common.cuh"
+#include "event_guard.hpp"
 #include "tile_registry.hpp"
 
 namespace sched {
@@ -593,6 +594,54 @@ int stage_tables(const DevParams &dp, const std::vector<unsigned char> &blob, vo
   return SCHED_OK;
 }
 
+// device unrank (+ successor walk) of a batch of indices (sched_unrank_device)
+__global__ void __launch_bounds__(256) k_unrank(const DevParams p, const u64 *idx, u64 n, u64 advance,
+                                                int8_t *gout, int8_t *lout) {
+  extern __shared__ __align__(16) unsigned char sm[];
+  stage_blob(sm, p);
+  const Tables tb = tables_at(sm, p);
+  for (u64 t = blockIdx.x * (u64)blockDim.x + threadIdx.x; t < n; t += (u64)gridDim.x * blockDim.x) {
+    int8_t *g = gout + t * p.n, *l = lout + t * p.n;
+    const u64 i0 = idx[t];
+    LaneCfg c;
+    if (i0 >= tb.W[p.root] || !dev_unrank(tb, p, i0, c) || (advance && !dev_advance(tb, p, c, advance))) {
+      g[0] = -1;
+      continue;
+    }
+    // level digits of residue v, base L, most significant = client 0 / group 0
+    const int nd = p.scope == SCHED_PER_CLIENT ? p.n : c.k;
+    int8_t dig[kMaxN];
+    u64 v = c.v;
+    for (int d = nd - 1; d >= 0; d--) {
+      dig[d] = (int8_t)(v % (u64)p.L);
+      v /= (u64)p.L;
+    }
+    for (int i = 0; i < p.n; i++) {
+      g[i] = c.a[i];
+      l[i] = p.scope == SCHED_PER_CLIENT ? dig[i] : dig[c.a[i]];
+    }
+  }
+}
+
+int launch_unrank(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, const uint64_t *d_idx, uint64_t n,
+                  uint64_t advance, int8_t *gout, int8_t *lout) {
+  const WsLayout L = layout(dp);
+  if (ws_bytes < L.total || ((uintptr_t)d_ws & 255)) return SCHED_E_WORKSPACE;
+  if (n == 0) return SCHED_OK;
+  unsigned char *ws = (unsigned char *)d_ws;
+  cudaStream_t st = (cudaStream_t)stream;
+  dp.blob = ws + L.blob;
+  const size_t smem = (dp.blob_bytes + 15) & ~15u;
+  CK(cudaFuncSetAttribute(k_unrank, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  int dev = 0, nsm = 0;
+  CK(cudaGetDevice(&dev));
+  CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
+  const int grid = (int)std::min<uint64_t>((n + 255) / 256, (uint64_t)nsm * 4);
+  k_unrank<<<grid, 256, smem, st>>>(dp, (const u64 *)d_idx, n, advance, gout, lout);
+  CK(cudaGetLastError());
+  return SCHED_OK;
+}
+
 int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, LaunchInfo *info,
                   std::vector<BestRec> *best, std::vector<CandRec> *pareto, uint64_t *ctr_out) {
   const WsLayout L = layout(dp);
@@ -614,10 +663,9 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   CK(cudaGetDevice(&dev));
   CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
 
-  cudaEvent_t e0, e1, e2;
-  CK(cudaEventCreate(&e0));
-  CK(cudaEventCreate(&e1));
-  CK(cudaEventCreate(&e2));
+  EventGuard<3> ev;  // destroyed on every return path
+  if (!ev.create()) return SCHED_E_CUDA;
+  cudaEvent_t e0 = ev[0], e1 = ev[1], e2 = ev[2];
   CK(cudaEventRecord(e0, st));
   int grid = 0, path = 0, launches = 0, passes = 0;
   uint64_t d2h = 0;
@@ -769,9 +817,6 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   info->d2h_bytes = d2h;
   for (int k = 0; k < kCtrN; k++) ctr_out[k] = ctr[k];
   ctr_out[kCtrFront] = nfront;
-  cudaEventDestroy(e0);
-  cudaEventDestroy(e1);
-  cudaEventDestroy(e2);
   if (nfront > kFrontCap) return SCHED_E_CAPACITY;
   return SCHED_OK;
 }

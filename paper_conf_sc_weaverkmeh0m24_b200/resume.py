@@ -19,6 +19,7 @@ import dataclasses
 import hashlib
 import json
 import os
+import warnings
 
 import numpy as np
 
@@ -115,17 +116,24 @@ def search_resumable(sched, profile, q, path: str, n_windows: int = 64, max_wind
     fp = fingerprint(profile, q)
     total = count(q)
     done = load(path, fp)
-    resumed = len(done)
     search = search_fn if search_fn is not None else (lambda qw: sched.search(qw, pareto_cap=pareto_cap))
     new = 0
     wins = windows_of(total, n_windows, align)
+    # only records of the current window split count as resumed; records of
+    # another split (n_windows / align changed) are ignored, not merged
+    resumed = sum(1 for w in wins if w in done)
+    stale = len(done) - resumed
+    if stale:
+        warnings.warn(f"{path}: {stale} checkpoint record(s) of another window split "
+                      f"(n_windows={n_windows}, align={align} now) are ignored", RuntimeWarning)
     for lo, hi in wins:
         if (lo, hi) in done:
             continue
         if max_windows is not None and new >= max_windows:
             return None
         res = search(q.with_range(lo, hi))
-        rec = {"fp": fp, "lo": lo, "hi": hi, "n_configs": int(res.stats["n_configs"]),
+        rec = {"fp": fp, "lo": lo, "hi": hi, "n_windows": n_windows, "align": align,
+               "n_configs": int(res.stats["n_configs"]),
                "n_feasible": int(res.stats["n_feasible"]),
                "best": [pick_to_json(b) for b in res.best],
                "pareto": [pick_to_json(p) for p in res.pareto]}
@@ -144,4 +152,4 @@ def search_resumable(sched, profile, q, path: str, n_windows: int = 64, max_wind
     best, par = merge(rank_best, rank_par, nw, pareto_cap)
     return best, par, {"n_configs": sum(r["n_configs"] for r in recs),
                        "n_feasible": sum(r["n_feasible"] for r in recs),
-                       "windows": len(recs), "resumed": resumed}
+                       "windows": len(recs), "resumed": resumed, "stale": stale}

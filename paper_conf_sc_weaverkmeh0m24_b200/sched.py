@@ -34,7 +34,7 @@ UINT64_MAX = (1 << 64) - 1
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
            "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score", "sched_heuristic",
            "sched_strerror", "sched_version", "sched_dp_workspace_size", "sched_front_dp",
-           "sched_split_workspace_size", "sched_search_splits"]
+           "sched_split_workspace_size", "sched_search_splits", "sched_unrank_device"]
 
 
 class SchedError(RuntimeError):
@@ -227,6 +227,14 @@ class Scheduler:
         return SearchResult(rc, [best[w] for w in range(nw)], [par[k] for k in range(npv)],
                             stats.as_dict())
 
+    def dp_workspace(self, q):
+        """A device workspace sized for sched_front_dp of q (caller-owned)."""
+        import torch
+        n = C.c_size_t()
+        _check(lib().sched_dp_workspace_size(self._h, C.byref(self.cquery(q)), C.byref(n)),
+               "sched_dp_workspace_size")
+        return torch.empty(n.value, dtype=torch.uint8, device="cuda")
+
     def front_dp(self, q, workspace=None, stream=None, front_cap=4096):
         """Exact Pareto front and per-weight optimum of the whole space by the
         device subset DP (sched_front_dp).  Returns (status, best[W], front,
@@ -294,6 +302,24 @@ class Scheduler:
         _check(lib().sched_heuristic(self._h, C.byref(self.cquery(q)), pr, w, a, lv, C.byref(idx), C.byref(out)),
                "sched_heuristic")
         return [a[i] for i in range(q.n)], [lv[i] for i in range(q.n)], idx.value, out
+
+    def unrank_device(self, q, indices, advance=0, workspace=None, stream=None):
+        """Device unrank (+ `advance` successor steps) of a uint64 tensor of
+        indices (sched_unrank_device).  Returns (group_of, level_of) int8
+        device tensors [n][q.n]; rows of out-of-range indices have
+        group_of[:, 0] = -1."""
+        import torch
+        idx = indices.to(device="cuda", dtype=torch.int64).contiguous()
+        n = idx.numel()
+        g = torch.empty((n, q.n), dtype=torch.int8, device="cuda")
+        lv = torch.empty((n, q.n), dtype=torch.int8, device="cuda")
+        ws = workspace if workspace is not None else self.workspace(q)
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        _check(lib().sched_unrank_device(self._h, C.byref(self.cquery(q)), C.c_void_p(idx.data_ptr()),
+                                         C.c_uint64(n), C.c_uint64(advance), C.c_void_p(g.data_ptr()),
+                                         C.c_void_p(lv.data_ptr()), C.c_void_p(ws.data_ptr()),
+                                         C.c_size_t(ws.numel()), C.c_void_p(st)), "sched_unrank_device")
+        return g, lv
 
     def score(self, q, index, w=0) -> Pick:
         out = Pick()

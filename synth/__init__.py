@@ -2,5 +2,5 @@
 
 Holds no scheduler arithmetic (see profiles.py docstring).
 """
-from .profiles import Profile, make_profile, table_iii_combo1, TABLE_II  # noqa: F401
+from .profiles import Profile, make_profile, requeue, table_iii_combo1, TABLE_II  # noqa: F401
 from .configs import Query, CONFIGS, config, PER_CLIENT, PER_GPU  # noqa: F401

@@ -281,3 +281,88 @@ def test_no_device_no_fallback():
                                      C.byref(npar), None)
     assert rc == S.sched.SCHED_E_NODEVICE
     assert S.lib().sched_strerror(S.sched.SCHED_E_NODEVICE)
+
+
+@pytest.mark.parametrize("scope", [PER_GPU, PER_CLIENT])
+def test_rank_rejects_out_of_range_groups_and_levels(scope):
+    """sched_rank validates every group id / level digit before using it as
+    an index (a group id >= 32 once wrote past a stack buffer)."""
+    q = Query(6, 4, 6, (25, 50, 75, 100), scope, ())
+    for a, lv in [([0, 40, 0, 1, 1, 2], [0] * 6), ([0, -1, 0, 1, 1, 2], [0] * 6),
+                  ([0, 1, 2, 3, 4, 0], [0] * 6),            # group 4 >= G = 4
+                  ([0, 0, 1, 1, 2, 2], [0, 0, 1, 1, 4, 4]),   # level digit 4 >= L
+                  ([0, 0, 1, 1, 2, 2], [0, 0, 1, 1, -1, -1]),
+                  ([0, 127, 0, 0, 0, 0], [0] * 6)]:
+        with pytest.raises(S.SchedError) as e:
+            S.rank(q, a, lv)
+        assert e.value.status == S.sched.SCHED_E_INVALID
+    assert S.rank(q, [0, 0, 1, 1, 2, 2], [1, 1, 2, 2, 3, 3] if scope == PER_GPU else [1, 2, 3, 0, 1, 2]) >= 0
+
+
+def _heuristic_cases():
+    rnd = random.Random(2024)
+    cases = []
+    for k in range(220):
+        n = rnd.randint(2, 12)
+        g = rnd.randint(1, 8)
+        c = rnd.randint(1, n)
+        lv = tuple(sorted(rnd.sample((25, 50, 75, 100), rnd.randint(1, 4))))
+        scope = rnd.choice((PER_GPU, PER_CLIENT))
+        if scope == PER_CLIENT and n > 9:
+            scope = PER_GPU
+        arch = None
+        if k % 5 == 0:   # memory-heavy mixes (WarpX, BerkeleyGW rows) exercise criterion 3
+            arch = [rnd.choice((2, 11, 12, 0, 3, 5)) for _ in range(n)]
+        cases.append((k, n, g, c, lv, scope, arch))
+    return cases
+
+
+def test_heuristic_equals_oracle_transcription():
+    """N2 parity: sched_heuristic returns exactly O6's schedule
+    (oracle/heuristic.py, criteria 1-4 of PAPER.md L89-L92, reading R25) --
+    group_of, level_of, index and fp64 score, or both report no schedule --
+    on 220 seeded queues x both priorities (n = 2..12, G = 1..8, every C,
+    level subsets, both scopes, memory-heavy mixes)."""
+    from oracle import heuristic as H
+    W2 = ((1, 1), (1, 0), (0, 1))
+    n_sched = n_none = 0
+    for k, n, g, c, lv, scope, arch in _heuristic_cases():
+        prof = make_profile(n, levels=(25, 50, 75, 100), seed=900 + k, archetypes=arch)
+        q = Query(n, g, c, lv, scope, W2, True)
+        sch = S.Scheduler(prof)
+        for pr in ("throughput", "energy"):
+            w = k % 3
+            ref = H.heuristic(prof, q, pr, w=w)
+            if ref is None:
+                with pytest.raises(S.SchedError) as e:
+                    sch.heuristic(q, pr, w)
+                assert e.value.status == S.sched.SCHED_E_INFEASIBLE
+                n_none += 1
+                continue
+            a, lvl, idx, pick = sch.heuristic(q, pr, w)
+            assert (a, lvl, idx) == (ref["rgs"], ref["level_of"], ref["index"]), (k, pr)
+            assert bool(pick.valid) == ref["feasible"]
+            if ref["feasible"]:
+                assert (pick.makespan_s, pick.energy_j, pick.score64) == (ref["T"], ref["E"], ref["score64"])
+            n_sched += 1
+        sch.close()
+    assert n_sched >= 250 and n_none >= 5
+
+
+@pytest.mark.parametrize("name", list(CONFIGS))
+def test_heuristic_equals_oracle_transcription_configs(name):
+    from oracle import heuristic as H
+    prof, q = config(name)
+    sch = S.Scheduler(prof)
+    for pr in ("throughput", "energy"):
+        for w in range(len(q.weights)):
+            ref = H.heuristic(prof, q, pr, w=w)
+            if ref is None:
+                with pytest.raises(S.SchedError):
+                    sch.heuristic(q, pr, w)
+                continue
+            a, lvl, idx, pick = sch.heuristic(q, pr, w)
+            assert (a, lvl, idx) == (ref["rgs"], ref["level_of"], ref["index"])
+            assert bool(pick.valid) == ref["feasible"]
+            if ref["feasible"]:
+                assert pick.score64 == ref["score64"]

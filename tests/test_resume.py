@@ -91,6 +91,19 @@ def test_torn_line_and_other_search_ignored(tmp_path):
     _same(out, oracle.search(prof, q))
 
 
+def test_changed_window_split_not_counted_as_resumed(tmp_path):
+    """Records of another window split (n_windows / align changed between
+    runs) are neither merged nor counted as resumed, and a warning names them."""
+    prof, q = _case()
+    ck = str(tmp_path / "ck.jsonl")
+    fn = _oracle_search_fn(prof, len(q.weights))
+    R.search_resumable(None, prof, q, ck, n_windows=4, align=64, max_windows=2, search_fn=fn)
+    with pytest.warns(RuntimeWarning, match="another window split"):
+        out = R.search_resumable(None, prof, q, ck, n_windows=7, align=32, search_fn=fn)
+    assert out[2]["resumed"] == 0 and out[2]["stale"] == 2
+    _same(out, oracle.search(prof, q))
+
+
 def test_truncated_window_raises_coverage_error(tmp_path):
     """Fault injection: a window search that silently scores fewer
     configurations than its range must not produce an 'optimum'."""
