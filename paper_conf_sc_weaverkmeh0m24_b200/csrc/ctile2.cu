@@ -1,0 +1,48 @@
+// ctile2.cu -- eligibility and launch of the group-table PER_CLIENT tile
+// kernel (search_ctile2.cuh, kernel_path 6): PER_CLIENT scope, L = 4,
+// 6 <= n <= 15, groups of <= 4 clients (C <= 4), G <= 8, canonical model or
+// POWER_CAP (E = sum_g E_g, level-independent feasibility).
+#include "search_ctile2.cuh"
+
+namespace sched {
+
+static size_t ctile2_smem(const DevParams &dp) {
+  return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(C2Warp) * kC2Warps + sizeof(BestRec) * kC2Warps * kMaxW;
+}
+
+bool ctile2_eligible(DevParams &dp, TileLaunch *tl) {
+  if (dp.scope != SCHED_PER_CLIENT || dp.L != 4 || dp.n < 6 || dp.n > 15 || dp.g > 8) return false;
+  if (dp.c > 4) return false;  // groups of <= 4 clients: tables <= 836 entries
+  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE | SCHED_MODEL_TIME_SLICE)) return false;
+  if (ctile2_smem(dp) > 227 * 1024) return false;
+  tl->fn = dp.nw <= 1 ? ctile2_fn<1>() : dp.nw <= 2 ? ctile2_fn<2>() : dp.nw <= 4 ? ctile2_fn<4>() : ctile2_fn<8>();
+  tl->smem = ctile2_smem(dp);
+  return true;
+}
+
+cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                          cudaEvent_t e2, int *grid, bool fixed_units) {
+  cudaError_t err = cudaFuncSetAttribute(tl.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)tl.smem);
+  if (err != cudaSuccess) return err;
+  int occ = 0;
+  err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kC2Threads, tl.smem);
+  if (err != cudaSuccess) return err;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  *grid = std::min(4096, nsm * occ);
+  if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
+    const uint64_t range = dp.n_owned << dp.chunk_log2;
+    const uint64_t warps = (uint64_t)(*grid) * kC2Warps;
+    int ul = 12;
+    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 8) ul++;
+    dp.unit_log2 = ul;
+    dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
+    dp.unit_stride = 1;
+  }
+  void *args[] = {(void *)&dp};
+  cudaEventRecord(e1, st);
+  err = cudaLaunchKernel(tl.fn, *grid, kC2Threads, args, tl.smem, st);
+  cudaEventRecord(e2, st);
+  return err;
+}
+
+}  // namespace sched

@@ -513,10 +513,10 @@ __global__ void k_pareto_order(const DevParams p, const unsigned int *surv, cons
 
 // ------------------------------------------------------------ launcher
 namespace {
-// SCHED_KERNEL=generic|tile|dfs|sfx|ctile restricts the kernel choice (testing and
+// SCHED_KERNEL=generic|tile|dfs|sfx|ctile|ctile2 restricts the kernel choice (testing and
 // measurement of the individual paths); unset = the fastest eligible path.
 bool want_path(int path) {
-  static const char *names[] = {"generic", "tile", "dfs", "sfx", "dp", "ctile"};
+  static const char *names[] = {"generic", "tile", "dfs", "sfx", "dp", "ctile", "ctile2"};
   const char *e = std::getenv("SCHED_KERNEL");
   if (!e || !*e) return true;
   return std::strcmp(e, names[path]) == 0;
@@ -749,6 +749,9 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     if (want_path(1) && tile_eligible(dp, &tl)) {
       path = 1;
       CK(launch_tile(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
+    } else if (want_path(6) && ctile2_eligible(dp, &tl)) {
+      path = 6;
+      CK(launch_ctile2(dp, tl, nsm, st, e1, e2, &grid, pass == 0));
     } else if (want_path(5) && ctile_eligible(dp, &tl)) {
       path = 5;
       CK(launch_ctile(dp, tl, nsm, st, e1, e2, &grid, pass == 0));

@@ -155,6 +155,11 @@ __device__ __forceinline__ int ct_check(const DevParams &p, const Stair &stair, 
   }
   if (!need && !par) return 0;
   if (!have) exact(T64, E64);
+  // weights with b = 0 (F = X^a depends on T alone): a best with makespan
+  // <= T64 at a lower index cannot be replaced -- exact early reject
+#pragma unroll
+  for (int w = 0; w < WM; w++)
+    if ((need >> w & 1u) && p.wb[w] == 0 && lb[w].valid && T64 >= lb[w].t && idx > lb[w].idx) need &= ~(1u << w);
 #pragma unroll
   for (int w = 0; w < WM; w++) {
     if (need >> w & 1u) {

@@ -115,7 +115,6 @@ static __device__ __noinline__ void sfx_check(const DevParams &p, const Stair &s
   }
   const bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(T, p.tlb_scale_f), E);
   if (!need && !par) return;
-  cold->nref++;
   const GroupRec *gtab = (const GroupRec *)p.gtab;
   double T64 = 0.0, E64 = 0.0;
   for (int g = 0; g < kc; g++) {
@@ -124,6 +123,16 @@ static __device__ __noinline__ void sfx_check(const DevParams &p, const Stair &s
     T64 = fmax(T64, r.t64);
     E64 = __dadd_rn(E64, r.e64);
   }
+  // weights with b = 0 (F = X^a depends on T alone): a best with makespan
+  // <= T64 at a lower index cannot be replaced (F <= its F, index higher) --
+  // exact early reject that stops the (1,0) tie flood
+#pragma unroll
+  for (int w = 0; w < kMaxW; w++)
+    if (w < p.nw && (need >> w & 1u) && p.wb[w] == 0 && cold->lb[w].valid && T64 >= cold->lb[w].t &&
+        idx > cold->lb[w].idx)
+      need &= ~(1u << w);
+  if (!need && !par) return;
+  cold->nref++;
 #pragma unroll
   for (int w = 0; w < kMaxW; w++) {
     if (w < p.nw && (need >> w & 1u)) {

@@ -23,30 +23,35 @@ namespace sched {
 
 // ---- compile-time product-metric sets: q_s = (T/T_seq)^a (E/E_seq)^b ----
 struct WS_P {  // Pareto only
+  static constexpr bool RT = false;
   static constexpr int N = 0;
   __host__ __device__ static constexpr int A(int s) { return 0; }
   __host__ __device__ static constexpr int B(int s) { return 0; }
   __device__ static __forceinline__ void q(float, float, float *) {}
 };
 struct WS_11 {
+  static constexpr bool RT = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 1; }
   __host__ __device__ static constexpr int B(int s) { return 1; }
   __device__ static __forceinline__ void q(float T, float E, float *o) { o[0] = E * T; }
 };
 struct WS_10 {
+  static constexpr bool RT = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 1; }
   __host__ __device__ static constexpr int B(int s) { return 0; }
   __device__ static __forceinline__ void q(float T, float, float *o) { o[0] = T; }
 };
 struct WS_01 {
+  static constexpr bool RT = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 0; }
   __host__ __device__ static constexpr int B(int s) { return 1; }
   __device__ static __forceinline__ void q(float, float E, float *o) { o[0] = E; }
 };
 struct WS_11_21 {  // c4: [T x E], [T x T x E]
+  static constexpr bool RT = false;
   static constexpr int N = 2;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : 2); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 1 : 1); }
@@ -56,6 +61,7 @@ struct WS_11_21 {  // c4: [T x E], [T x T x E]
   }
 };
 struct WS_C1 {  // (1,0) (0,1) (1,1) (2,1)
+  static constexpr bool RT = false;
   static constexpr int N = 4;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : (s == 1 ? 0 : (s == 2 ? 1 : 2))); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 0 : (s == 1 ? 1 : (s == 2 ? 1 : 1))); }
@@ -67,6 +73,7 @@ struct WS_C1 {  // (1,0) (0,1) (1,1) (2,1)
   }
 };
 struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
+  static constexpr bool RT = false;
   static constexpr int N = 7;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : (s == 1 ? 3 : (s == 2 ? 2 : (s == 3 ? 1 : (s == 4 ? 1 : (s == 5 ? 1 : 0)))))); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 0 : (s == 1 ? 1 : (s == 2 ? 1 : (s == 3 ? 1 : (s == 4 ? 2 : (s == 5 ? 3 : 1)))))); }
@@ -82,10 +89,33 @@ struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
   }
 };
 
+// Any W <= 8 product metrics with the exponents read at run time
+// (p.wa / p.wb, "different product metrics"): the per-tile
+// corner screen evaluates q_w = T^a E^b by repeated multiplication; the
+// lane's running thresholds live in its shared-memory row (thr_sm), not in
+// registers, so the tile loop's register footprint is that of WS_11_21.
+struct WS_RT {
+  static constexpr int N = kMaxW;
+  static constexpr bool RT = true;
+  __host__ __device__ static constexpr int A(int) { return 0; }
+  __host__ __device__ static constexpr int B(int) { return 0; }
+  __device__ static __forceinline__ void q(float, float, float *) {}
+};
+
+// q_s = (T/T_seq)^a (E/E_seq)^b for query weight s, run-time exponents
+__device__ __forceinline__ float rt_q(const DevParams &p, int s, float T, float E) {
+  float q = 1.f;
+  for (int i = 0; i < p.wa[s]; i++) q *= T;
+  for (int i = 0; i < p.wb[s]; i++) q *= E;
+  return q;
+}
+
 
 struct WarpPart {
   LaneCfg cfg;
   u64 base;
+  u64 ncfg, nfeas;   // configurations scored / feasible (lane 0 counts; shared memory, not registers)
+  u64 sver;          // staircase insertion-log position this warp has applied
   float gt[kTileMaxG * 4], ge[kTileMaxG * 4];
   double g64[kTileMaxG * 4];
   double ge64[kTileMaxG * 4];  // exact canonical fp64 E_g per (group, level)
@@ -116,6 +146,41 @@ __device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParam
   return false;
 }
 
+// bit s set: weight s has b = 0 (F = X^a depends on T alone) and the lane's
+// best for it has T <= T64 and a lower index than idx: configurations with
+// makespan >= T64 and index >= idx have F <= that best's F (rounding is
+// monotone) and a higher index, so none of them can replace it
+template <class WS>
+__device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec *lb, unsigned mask, double T64,
+                                              u64 idx) {
+  unsigned out = 0;
+  if constexpr (WS::RT) {
+    for (int s = 0; s < p.nw; s++)
+      if ((mask >> s & 1u) && p.wb[s] == 0 && lb[s].valid && T64 >= lb[s].t && idx > lb[s].idx) out |= 1u << s;
+  } else {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++)
+      if (WS::B(s) == 0 && (mask >> s & 1u) && lb[s].valid && T64 >= lb[s].t && idx > lb[s].idx)
+        out |= 1u << s;
+  }
+  return out;
+}
+
+// any weight with b = 0 among mask
+template <class WS>
+__device__ __forceinline__ bool b0_any(const DevParams &p, unsigned mask) {
+  if constexpr (WS::RT) {
+    for (int s = 0; s < p.nw; s++)
+      if ((mask >> s & 1u) && p.wb[s] == 0) return true;
+    return false;
+  } else {
+    bool any = false;
+#pragma unroll
+    for (int s = 0; s < WS::N; s++) any |= WS::B(s) == 0 && (mask >> s & 1u);
+    return any;
+  }
+}
+
 // One configuration of the current partition (level digits dig[0..k-1],
 // exact T64, fp32 T/E): per-weight screen against the lane's thresholds
 // (thr: shared-memory copy), Pareto screen, fp64 refine, record.  Out of
@@ -125,7 +190,13 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
                                          const WarpPart &wp, float *thr, BestRec *lb, u64 idx,
                                          const int *dig, float T, float E, double T64) {
   unsigned need = 0;
-  if constexpr (WS::N > 0) {
+  if constexpr (WS::RT) {
+    for (int s = 0; s < p.nw; s++) {
+      const float q = rt_q(p, s, T, E);
+      if (q <= fminf(thr[s], q) * p.mul[s]) need |= 1u << s;
+      thr[s] = fminf(thr[s], q);
+    }
+  } else if constexpr (WS::N > 0) {
     float q[WS::N];
     WS::q(T, E, q);
 #pragma unroll
@@ -134,6 +205,10 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
       thr[s] = fminf(thr[s], q[s]);
     }
   }
+  // weights with b = 0 (F = X^a, X = T_seq / T): exact early reject against
+  // the lane's best (b0_beaten) -- stops the tie flood of (1,0), where every
+  // configuration sharing the optimum's bottleneck group ties it
+  need &= ~b0_beaten<WS>(p, lb, need, T64, idx);
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
   // fp64 canonical re-score from the exact group tuples: T = max_g T_g (exact),
@@ -145,7 +220,8 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
 #pragma unroll
     for (int s = 0; s < WS::N; s++) {
       if (need >> s & 1u) {
-        const double F = objective64(p, T64r, E64, WS::A(s), WS::B(s));
+        const double F = WS::RT ? objective64(p, T64r, E64, p.wa[s], p.wb[s])
+                                : objective64(p, T64r, E64, WS::A(s), WS::B(s));
         BestRec &b = lb[s];
         if (!b.valid || better(F, idx, b.f, b.idx)) {
           b.f = F;
@@ -184,7 +260,9 @@ __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, c
       E += wp.ge[b * 4 + dig[b]];
       T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
-    if constexpr (WS::N > 0) {
+    if constexpr (WS::RT) {
+      for (int s = 0; s < p.nw; s++) thr[s] = fminf(thr[s], rt_q(p, s, T, E));
+    } else if constexpr (WS::N > 0) {
       float q[WS::N];
       WS::q(T, E, q);
 #pragma unroll
@@ -247,6 +325,23 @@ static __device__ __noinline__ double tile_corner64(const WarpPart &wp, uint32_t
   return t;
 }
 
+// the lane's thresholds: registers (compile-time sets) <-> its shared-memory
+// row for the out-of-line slow paths; WS_RT keeps them in shared memory only
+template <class WS>
+__device__ __forceinline__ void thr_to_sm(const Thr<WS> &thr, float *thr_sm) {
+  if constexpr (!WS::RT) {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+  }
+}
+template <class WS>
+__device__ __forceinline__ void thr_from_sm(Thr<WS> &thr, const float *thr_sm) {
+  if constexpr (!WS::RT) {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+  }
+}
+
 // All level vectors v in [v0, v1) of the current partition (L = 4).
 // k >= 5: lane = (h, digit of group k-5, digit of group k-4); the warp loop
 // runs over j = digit strings of groups 0..k-6, two per step (h selects);
@@ -257,11 +352,9 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                                  uint32_t v0, uint32_t v1, int lane) {
   const int k = wp.cfg.k;
   if (k < 5) {
-#pragma unroll
-    for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+    thr_to_sm<WS>(thr, thr_sm);
     const int r = edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
-#pragma unroll
-    for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+    thr_from_sm<WS>(thr, thr_sm);
     return r;
   }
   const int nloop = 1 << (2 * (k - 5));
@@ -302,14 +395,12 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     const float2 lp = wp.lp[j];
     const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
     if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-#pragma unroll
-      for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+      thr_to_sm<WS>(thr, thr_sm);
       nref += edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
-#pragma unroll
-      for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+      thr_from_sm<WS>(thr, thr_sm);
       continue;
     }
-    bool hit = false;
+    unsigned hitm = 0;
     float cE, cT;
     if constexpr (WS::N > 0) {
       // every configuration's (T, E), min-reduced over the tile: the tile's
@@ -332,10 +423,16 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
           }
         }
       }
-      float mq[WS::N];
-      WS::q(mT, mE, mq);
+      if constexpr (WS::RT) {
+        for (int s = 0; s < p.nw; s++)
+          if (rt_q(p, s, mT, mE) <= thr_sm[s] * p.mul[s]) hitm |= 1u << s;
+      } else {
+        float mq[WS::N];
+        WS::q(mT, mE, mq);
 #pragma unroll
-      for (int s = 0; s < WS::N; s++) hit |= mq[s] <= thr.v[s] * thr.m[s];
+        for (int s = 0; s < WS::N; s++)
+          if (mq[s] <= thr.v[s] * thr.m[s]) hitm |= 1u << s;
+      }
       cE = mE;
       cT = mT;
     } else {  // Pareto only: per-configuration E, min-reduced
@@ -352,15 +449,19 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         }
       }
     }
+    double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
+    if (hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
+      c64 = tile_corner64(wp, vt);
+      hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+    }
+    const bool hit = hitm != 0;
     bool par = false;
     if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
-      par = !stair_dominated(stair, p, tile_corner64(wp, vt), cE);
+      par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
     if (hit || par) {
-#pragma unroll
-      for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
+      thr_to_sm<WS>(thr, thr_sm);
       nref += tile_slow<WS>(tb, p, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
-#pragma unroll
-      for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+      thr_from_sm<WS>(thr, thr_sm);
     }
   }
   __syncwarp();
@@ -378,7 +479,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   WarpPart *wps = (WarpPart *)(after + kStairSmem);
   WarpPart &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kTileWarps);
-  float *thr_sm = (float *)(red + kTileWarps * kMaxW) + threadIdx.x * kMaxW;
+  float *thr_sm = (float *)(red + kTileWarps * kMaxW) + threadIdx.x * (kMaxW + 1);  // odd row stride: no bank conflicts
   const GroupRec *gtab = (const GroupRec *)p.gtab;
   stair_init(stair);
   __syncthreads();
@@ -387,11 +488,21 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   BestRec lb[WS::N > 0 ? WS::N : 1];
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {
-    thr.v[s] = __int_as_float(0x7f800000);
-    thr.m[s] = s < WS::N ? p.mul[p.ws_perm[s]] : 1.f;
+    if constexpr (WS::RT) {
+      thr_sm[s] = __int_as_float(0x7f800000);
+    } else {
+      thr.v[s] = __int_as_float(0x7f800000);
+      thr.m[s] = s < WS::N ? p.mul[p.ws_perm[s]] : 1.f;
+    }
     best_init(lb[s]);
   }
-  u64 ncfg = 0, nfeas = 0, stair_ver = 0;
+  const int nws = WS::RT ? p.nw : WS::N;  // weights searched
+  if (lane == 0) {
+    wp.ncfg = 0;
+    wp.nfeas = 0;
+    wp.sver = 0;
+  }
+  __syncwarp();
   int nref = 0;
   const int ul = p.unit_log2, cl = p.chunk_log2;
 
@@ -407,10 +518,17 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     s = s > p.lo ? s : p.lo;
     e = e < p.hi ? e : p.hi;
     if (s >= e) continue;
+    if constexpr (WS::RT) {
+      for (int w = 0; w < nws; w++) thr_sm[w] = fminf(thr_sm[w], __uint_as_float(__ldcg(p.thr + w)));
+    } else {
 #pragma unroll
-    for (int w = 0; w < WS::N; w++) thr.v[w] = fminf(thr.v[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
+      for (int w = 0; w < WS::N; w++) thr.v[w] = fminf(thr.v[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
+    }
     if (p.want_pareto) {
-      stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
+      u64 sv = wp.sver;
+      stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
+      __syncwarp();
+      if (lane == 0) wp.sver = sv;
     }
     if (lane == 0) {
       dev_unrank(tb, p, s, wp.cfg);
@@ -420,8 +538,11 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     u64 ver_pref = p.want_pareto ? __ldcg(p.ctr + kCtrStairVer) : 0;  // stair_sync broadcasts lane 0's
     for (;;) {
       if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
-        stair_sync(stair, p, stair_ver, ver_pref);
+        u64 sv = wp.sver;
+        stair_sync(stair, p, sv, ver_pref);
         ver_pref = __ldcg(p.ctr + kCtrStairVer);  // consumed next partition: load latency off the path
+        __syncwarp();
+        if (lane == 0) wp.sver = sv;
       }
       const u64 base = wp.base;
       const uint32_t Pn = (uint32_t)wp.cfg.Pn;
@@ -441,8 +562,8 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
       }
       const bool feas = __ballot_sync(0xffffffffu, infeas) == 0u;
       if (lane == 0) {
-        ncfg += v1 - v0;
-        if (feas) nfeas += v1 - v0;
+        wp.ncfg += v1 - v0;
+        if (feas) wp.nfeas += v1 - v0;
       }
       __syncwarp();
       if (feas) nref += partition_configs<WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
@@ -458,10 +579,12 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     }
 #pragma unroll
     for (int w = 0; w < WS::N; w++) {
-      float t = thr.v[w];
+      if (w >= nws) break;
+      float t = WS::RT ? thr_sm[w] : thr.v[w];
 #pragma unroll
       for (int o = 16; o; o >>= 1) t = fminf(t, __shfl_xor_sync(0xffffffffu, t, o));
-      thr.v[w] = t;
+      if constexpr (WS::RT) thr_sm[w] = t;
+      else thr.v[w] = t;
       if (lane == 0 && t < __uint_as_float(__ldcg(p.thr + p.ws_perm[w])))
         atomicMin(p.thr + p.ws_perm[w], __float_as_uint(t));
     }
@@ -469,23 +592,21 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   // ---- reductions ----
   u64 nref64 = (u64)nref;
 #pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    ncfg += __shfl_xor_sync(0xffffffffu, ncfg, o);
-    nfeas += __shfl_xor_sync(0xffffffffu, nfeas, o);
-    nref64 += __shfl_xor_sync(0xffffffffu, nref64, o);
-  }
+  for (int o = 16; o; o >>= 1) nref64 += __shfl_xor_sync(0xffffffffu, nref64, o);
+  __syncwarp();
   if (lane == 0) {
-    atomicAdd(p.ctr + kCtrConfigs, ncfg);
-    atomicAdd(p.ctr + kCtrFeasible, nfeas);
+    atomicAdd(p.ctr + kCtrConfigs, wp.ncfg);
+    atomicAdd(p.ctr + kCtrFeasible, wp.nfeas);
     atomicAdd(p.ctr + kCtrRefined, nref64);
   }
 #pragma unroll
   for (int w = 0; w < WS::N; w++) {
+    if (w >= nws) break;
     warp_best(lb[w]);
     if (lane == 0) red[warp * kMaxW + w] = lb[w];
   }
   __syncthreads();
-  if (threadIdx.x < WS::N) {
+  if ((int)threadIdx.x < nws) {
     const int w = threadIdx.x;
     BestRec b = red[w];
     for (int k = 1; k < kTileWarps; k++) {

@@ -35,12 +35,17 @@ static const void *tile_pick_ws(DevParams *dp) {
   TRY(WS_01)
   TRY(WS_11_21)
 #undef TRY
+  // any other 1 <= W <= 8: run-time exponents (query order)
+  if (dp->nw >= 1 && dp->nw <= kMaxW) {
+    for (int s = 0; s < dp->nw; s++) dp->ws_perm[s] = s;
+    return tile_fn<L, WS_RT>();
+  }
   return nullptr;
 }
 
 size_t tile_smem_bytes(const DevParams &dp) {
   return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(WarpPart) * kTileWarps +
-         sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * kMaxW;
+         sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * (kMaxW + 1);
 }
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {

@@ -16,6 +16,7 @@ struct WS_01;
 struct WS_11_21;
 struct WS_SWEEP;
 struct WS_C1;
+struct WS_RT;
 
 template <int L, class WS>
 const void *tile_fn();
@@ -42,6 +43,9 @@ bool tile_eligible(DevParams &dp, TileLaunch *tl);
 bool dfs_eligible(DevParams &dp, TileLaunch *tl);
 bool sfx_eligible(DevParams &dp, TileLaunch *tl);
 bool ctile_eligible(DevParams &dp, TileLaunch *tl);
+bool ctile2_eligible(DevParams &dp, TileLaunch *tl);
+cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
+                          cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_ctile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
                          cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,

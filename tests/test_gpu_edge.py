@@ -84,7 +84,7 @@ CASES = {
     "dup_c4_tile": (_dup_c4, 1), "dup_combo8_tile": (_dup_combo8, 1), "mem_c4_tile": (_mem_c4, 1),
     "dup_c5_sfx": (_dup_c5, 3), "mem_c5_sfx": (_mem_c5, 3),
     "dup_c2_ctile": (lambda: _c2like("dup"), 5), "mem_c2_ctile": (lambda: _c2like("mem"), 5),
-    "dup_c3client_ctile": (lambda: _c3client("dup"), 5), "mem_c3client_ctile": (lambda: _c3client("mem"), 5),
+    "dup_c3client_ctile": (lambda: _c3client("dup"), 6), "mem_c3client_ctile": (lambda: _c3client("mem"), 6),
 }
 
 

@@ -282,14 +282,18 @@ def test_maximum_sizes_windows(n, g, c, levels, scope):
     (7, 4, 2, ((2, 1), (1, 3)), True, 0, 14),
     (6, 6, 6, (), True, 0, 15),                        # Pareto only, many groups
 ])
-def test_client_tile_kernel_path(n, g, c, ws, pareto, model, seed):
-    """PER_CLIENT, L = 4 spaces on the PER_CLIENT tile kernel (kernel_path 5):
+@pytest.mark.parametrize("kernel", ["ctile", "auto"])
+def test_client_tile_kernel_path(n, g, c, ws, pareto, model, seed, kernel, monkeypatch):
+    """PER_CLIENT, L = 4 spaces on the PER_CLIENT tile kernels (kernel_path 5;
+    auto picks the group-table kernel, path 6, when groups have <= 4 clients):
     full space and ragged windows bitwise against the oracle."""
+    if kernel != "auto":
+        monkeypatch.setenv("SCHED_KERNEL", kernel)
     prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
     q = Query(n, g, c, (25, 50, 75, 100), PER_CLIENT, ws, pareto, model=model, power_cap=150.0)
     sch = S.Scheduler(prof)
     res = sch.search(q)
-    assert res.stats["kernel_path"] == 5
+    assert res.stats["kernel_path"] == (5 if kernel == "ctile" or c > 4 else 6)
     check(res, oracle.search(prof, q), q)
     tot = S.count(q)
     for lo, hi in ((1000, 70_001), (tot // 2 - 4097, tot // 2 + 33_333), (tot - 50_000, tot)):
