@@ -21,6 +21,7 @@
 
 #include "device_common.cuh"
 #include "event_guard.hpp"
+#include "finalize.hpp"
 #include "tile_registry.hpp"
 
 namespace sched {
@@ -462,54 +463,6 @@ __global__ void k_pareto_prefilter(const DevParams p, int ncand, unsigned int *s
   }
 }
 
-// stage 2: exact O(m^2) dominance among survivors (smem tiles); keep[s] = 1 if
-// on the front (one representative per distinct (T,E): the lowest index).
-__global__ void k_pareto_exact(const DevParams p, const unsigned int *surv, unsigned int *keep) {
-  __shared__ CandRec tile[256];
-  const int m = (int)(*(volatile unsigned long long *)(p.ctr + kCtrSurv));
-  const CandRec *cand = (const CandRec *)p.cand;
-  for (int base = blockIdx.x * blockDim.x; base < m; base += gridDim.x * blockDim.x) {
-    const int s = base + threadIdx.x;
-    CandRec me;
-    if (s < m) me = cand[surv[s]];
-    bool alive = s < m;
-    for (int t0 = 0; t0 < m; t0 += 256) {
-      __syncthreads();
-      if (t0 + threadIdx.x < m) tile[threadIdx.x] = cand[surv[t0 + threadIdx.x]];
-      __syncthreads();
-      const int nt = min(256, m - t0);
-      if (alive) {
-        for (int k = 0; k < nt; k++) {
-          const CandRec o = tile[k];
-          const bool dom = (o.t <= me.t && o.e <= me.e && (o.t < me.t || o.e < me.e)) ||
-                           (o.t == me.t && o.e == me.e && (o.idx < me.idx || (o.idx == me.idx && t0 + k < s)));
-          if (dom) {
-            alive = false;
-            break;
-          }
-        }
-      }
-    }
-    if (s < m) keep[s] = alive ? 1u : 0u;
-  }
-}
-
-// stage 3: order the front by T ascending (= X descending) into out[W ...]
-__global__ void k_pareto_order(const DevParams p, const unsigned int *surv, const unsigned int *keep,
-                               int out_cap) {
-  const int m = (int)(*(volatile unsigned long long *)(p.ctr + kCtrSurv));
-  const CandRec *cand = (const CandRec *)p.cand;
-  CandRec *out = (CandRec *)(p.out + sizeof(BestRec) * kMaxW);
-  for (int s = blockIdx.x * blockDim.x + threadIdx.x; s < m; s += gridDim.x * blockDim.x) {
-    if (!keep[s]) continue;
-    const CandRec me = cand[surv[s]];
-    int rank = 0;
-    for (int t = 0; t < m; t++)
-      if (keep[t] && cand[surv[t]].t < me.t) rank++;
-    if (rank < out_cap) out[rank] = me;
-    atomicAdd(p.ctr + kCtrFront, 1ull);
-  }
-}
 
 // ------------------------------------------------------------ launcher
 namespace {
@@ -542,7 +495,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, keep, out, gtab, total;
+  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, fin, out, gtab, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -564,7 +517,7 @@ WsLayout layout(const DevParams &dp) {
   L.slots = take(sizeof(BestRec) * kMaxW * (size_t)kMaxGrid);
   L.cand = take(sizeof(CandRec) * (size_t)dp.cand_cap);
   L.surv = take(4 * (size_t)dp.cand_cap);
-  L.keep = take(4 * (size_t)dp.cand_cap);
+  L.fin = take(finalize_bytes(dp.cand_cap));
   L.out = take(sizeof(BestRec) * kMaxW + sizeof(CandRec) * (size_t)kFrontCap);
   L.gtab = take(dp.gtab_ok ? sizeof(GroupRec) * ((size_t)dp.L << dp.n) : 0);
   L.total = (o + 255) / 256 * 256;
@@ -694,7 +647,11 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   DevParams dp_full = dp;
   const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
                     (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 20);  // >= 2^32 configs
-  for (int pass = seed ? 0 : 1; pass < 3; pass++) {
+  // passes: 0 seed (large searches), 1 full search, 2 re-run after a
+  // candidate-buffer overflow (unseeded: re-bucketed to the overflowing
+  // pass's front span with a fresh staircase; seeded: reseeded staircase),
+  // 3 reseeded re-run if 2 overflowed as well
+  for (int pass = seed ? 0 : 1; pass < 4; pass++) {
     dp = dp_full;
     if (pass == 0) {
       const int sl = seed_unit_log2();
@@ -705,7 +662,9 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     }
     passes++;
     int keep = pass == 0 ? 0 : (pass == 1 ? (seed ? 2 : 0) : 1);
-    const int ncand0 = pass == 1 && seed && dp.want_pareto ? (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap) : 0;
+    const bool span_rerun = pass == 2 && !seed && dp.want_pareto;  // dense front flooded coarse buckets
+    const int ncand0 = (pass == 1 && seed && dp.want_pareto) || span_rerun
+                           ? (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap) : 0;
     if (ncand0 > 0) {
       // Re-bucket the staircase to the span of the seed pass's front: about
       // 1024 buckets between its lowest T and the T of its lowest-E point,
@@ -729,7 +688,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
         dp_full.bucket_base = (uint32_t)std::max<int64_t>(0, base);
         dp.bucket_shift = dp_full.bucket_shift;
         dp.bucket_base = dp_full.bucket_base;
-        keep = 3;
+        keep = span_rerun ? 0 : 3;   // the re-run starts a fresh staircase in the finer buckets
       }
     }
     k_init<<<1, 256, 0, st>>>(dp, keep);
@@ -740,7 +699,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       CK(cudaGetLastError());
       launches++;
     }
-    if (pass == 2 && dp.want_pareto) {
+    if (pass >= 2 && keep == 1 && dp.want_pareto) {
       k_reseed<<<1, 1024, 0, st>>>(dp, (CandRec *)dp.out);
       CK(cudaGetLastError());
       launches++;
@@ -789,15 +748,16 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   }
   int ncand = (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap);
   if (dp.want_pareto && ncand > 0) {
-    unsigned int *surv = (unsigned int *)(ws + L.surv), *keep = (unsigned int *)(ws + L.keep);
+    // exact front: staircase prefilter, then sort + sweep (finalize.cu)
+    unsigned int *surv = (unsigned int *)(ws + L.surv);
     k_pareto_prefilter<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, ncand, surv);
     CK(cudaGetLastError());
-    k_pareto_exact<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, surv, keep);
-    CK(cudaGetLastError());
-    k_pareto_order<<<std::max(1, std::min(4 * nsm, (ncand + 255) / 256)), 256, 0, st>>>(dp, surv, keep,
-                                                                                        kFrontCap);
-    CK(cudaGetLastError());
-    launches += 3;
+    launches++;
+    unsigned long long nsurv = 0;
+    CK(cudaMemcpyAsync(&nsurv, dp.ctr + kCtrSurv, sizeof nsurv, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    d2h += sizeof nsurv;
+    CK(finalize_front(dp, ws + L.fin, finalize_bytes(dp.cand_cap), surv, (int)nsurv, kFrontCap, nsm, st, &launches));
   }
   CK(cudaMemcpyAsync(ctr, dp.ctr, sizeof ctr, cudaMemcpyDeviceToHost, st));
   best->resize(kMaxW);

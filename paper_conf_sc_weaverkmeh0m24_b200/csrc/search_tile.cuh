@@ -166,6 +166,21 @@ __device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec 
   return out;
 }
 
+// mask of the weights with b = 0
+template <class WS>
+__device__ __forceinline__ unsigned b0_mask(const DevParams &p) {
+  unsigned m = 0;
+  if constexpr (WS::RT) {
+    for (int s = 0; s < p.nw; s++)
+      if (p.wb[s] == 0) m |= 1u << s;
+  } else {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++)
+      if (WS::B(s) == 0) m |= 1u << s;
+  }
+  return m;
+}
+
 // any weight with b = 0 among mask
 template <class WS>
 __device__ __forceinline__ bool b0_any(const DevParams &p, unsigned mask) {
@@ -382,6 +397,22 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     Ct[m] = wp.gt[gc + m];
     Ce[m] = wp.ge[gc + m];
   }
+  // weights with b = 0 that no configuration of this partition can improve
+  // for this lane: the partition's exact min makespan (max over groups of the
+  // group's min over levels of the exact fp64 T_g) is >= the T of the lane's
+  // best and every index is higher (b0_beaten) -- then the tie flood of such
+  // weights (every configuration sharing the optimum's bottleneck group ties
+  // it) never reaches the per-tile exact corner
+  unsigned b0skip = 0;
+  {
+    const unsigned b0m = b0_mask<WS>(p);
+    if (b0m) {
+      double pc = 0.0;
+      for (int b = 0; b < k; b++)
+        pc = fmax(pc, fmin(fmin(wp.g64[b * 4], wp.g64[b * 4 + 1]), fmin(wp.g64[b * 4 + 2], wp.g64[b * 4 + 3])));
+      b0skip = b0_beaten<WS>(p, lb, b0m, pc, wp.base + v0);
+    }
+  }
   const float minTin = WS::N > 0 ? 0.f
                                  : fmaxf(fmaxf(fminf(fminf(At[0], At[1]), fminf(At[2], At[3])),
                                                fminf(fminf(Bt[0], Bt[1]), fminf(Bt[2], Bt[3]))),
@@ -449,6 +480,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         }
       }
     }
+    hitm &= ~b0skip;
     double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
     if (hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
       c64 = tile_corner64(wp, vt);

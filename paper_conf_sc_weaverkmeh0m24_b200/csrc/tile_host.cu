@@ -1,4 +1,6 @@
 // tile_host.cu -- weight-set matching and launch of the PER_GPU tile kernel.
+#include <cstdlib>
+
 #include "search_tile.cuh"
 
 namespace sched {
@@ -24,8 +26,12 @@ static bool ws_match(const DevParams &dp, int *perm) {
 template <int L>
 static const void *tile_pick_ws(DevParams *dp) {
   int perm[kMaxW];
+  // SCHED_TILE_RT=1 (measurement): the run-time-weight variant even where a
+  // compiled-in weight set matches
+  const char *rt = std::getenv("SCHED_TILE_RT");
+  const bool force_rt = rt && rt[0] == '1' && dp->nw >= 1;
 #define TRY(WS)                                                 \
-  if (ws_match<WS>(*dp, perm) && (WS::N > 0 || dp->want_pareto)) { \
+  if (!force_rt && ws_match<WS>(*dp, perm) && (WS::N > 0 || dp->want_pareto)) { \
     for (int s = 0; s < WS::N; s++) dp->ws_perm[s] = perm[s];     \
     return tile_fn<L, WS>();                                    \
   }
@@ -34,6 +40,8 @@ static const void *tile_pick_ws(DevParams *dp) {
   TRY(WS_10)
   TRY(WS_01)
   TRY(WS_11_21)
+  TRY(WS_C1)      // BASELINE configs[0]'s objectives: (1,0) (0,1) (1,1) (2,1)
+  TRY(WS_SWEEP)   // configs[4]'s sweep: (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
 #undef TRY
   // any other 1 <= W <= 8: run-time exponents (query order)
   if (dp->nw >= 1 && dp->nw <= kMaxW) {

@@ -18,6 +18,9 @@ SETS = {
     "eight": ((1, 0), (0, 1), (1, 1), (2, 1), (1, 2), (3, 1), (1, 3), (4, 4)),
     "pareto": (),
     "w11": ((1, 1),),
+    "w10": ((1, 0),),
+    "w10_01": ((1, 0), (0, 1)),
+    "w11_21_12": ((1, 1), (2, 1), (1, 2)),
 }
 
 ap = argparse.ArgumentParser()
