@@ -23,6 +23,13 @@
 
 namespace sched {
 
+// per-lane thresholds of the pair kernel: value and 1 + delta per weight slot
+template <class WS>
+struct DThr {
+  float v[WS::N > 0 ? WS::N : 1];
+  float m[WS::N > 0 ? WS::N : 1];
+};
+
 constexpr int kDfsMaxC = 4;
 constexpr int kDfsMaxG = 8;
 constexpr int kDfsThreads = 256;
@@ -223,7 +230,7 @@ __global__ void __launch_bounds__(kDfsThreads, 2) k_dfs(const DevParams p) {
   }
   __syncthreads();
 
-  Thr<WS> thr;
+  DThr<WS> thr;
   BestRec lb[WS::N > 0 ? WS::N : 1];
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {

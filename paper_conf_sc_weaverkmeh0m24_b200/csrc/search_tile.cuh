@@ -122,10 +122,13 @@ struct WarpPart {
   float2 lp[64];  // loop-prefix (max T, sum E) over groups 0..k-6, one entry per digit string
 };
 
+// The lane's running thresholds live in its shared-memory row (thr_sm, the
+// master copy, also used by the out-of-line slow paths); the tile screen
+// reads their products with 1 + delta from registers: one register per
+// weight (the c5 sweep's 7 weights: 7, not 14).
 template <class WS>
 struct Thr {
-  float v[WS::N > 0 ? WS::N : 1];
-  float m[WS::N > 0 ? WS::N : 1];  // 1 + delta of the weight in slot s (registers: no indexed param loads)
+  float vm[WS::N > 0 ? WS::N : 1];  // thr_sm[s] * (1 + delta of the weight in slot s)
 };
 
 // quick Pareto screen from fp32 values: tlb = certified lower bound of the
@@ -340,20 +343,13 @@ static __device__ __noinline__ double tile_corner64(const WarpPart &wp, uint32_t
   return t;
 }
 
-// the lane's thresholds: registers (compile-time sets) <-> its shared-memory
-// row for the out-of-line slow paths; WS_RT keeps them in shared memory only
+// after the lane's shared-memory thresholds changed: refresh the register
+// products (WS_RT screens from shared memory directly)
 template <class WS>
-__device__ __forceinline__ void thr_to_sm(const Thr<WS> &thr, float *thr_sm) {
+__device__ __forceinline__ void thr_from_sm(const DevParams &p, Thr<WS> &thr, const float *thr_sm) {
   if constexpr (!WS::RT) {
 #pragma unroll
-    for (int s = 0; s < WS::N; s++) thr_sm[s] = thr.v[s];
-  }
-}
-template <class WS>
-__device__ __forceinline__ void thr_from_sm(Thr<WS> &thr, const float *thr_sm) {
-  if constexpr (!WS::RT) {
-#pragma unroll
-    for (int s = 0; s < WS::N; s++) thr.v[s] = thr_sm[s];
+    for (int s = 0; s < WS::N; s++) thr.vm[s] = thr_sm[s] * p.mul[p.ws_perm[s]];
   }
 }
 
@@ -367,9 +363,8 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                                  uint32_t v0, uint32_t v1, int lane) {
   const int k = wp.cfg.k;
   if (k < 5) {
-    thr_to_sm<WS>(thr, thr_sm);
     const int r = edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
-    thr_from_sm<WS>(thr, thr_sm);
+    thr_from_sm<WS>(p, thr, thr_sm);
     return r;
   }
   const int nloop = 1 << (2 * (k - 5));
@@ -426,9 +421,8 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     const float2 lp = wp.lp[j];
     const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
     if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-      thr_to_sm<WS>(thr, thr_sm);
       nref += edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
-      thr_from_sm<WS>(thr, thr_sm);
+      thr_from_sm<WS>(p, thr, thr_sm);
       continue;
     }
     unsigned hitm = 0;
@@ -462,7 +456,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         WS::q(mT, mE, mq);
 #pragma unroll
         for (int s = 0; s < WS::N; s++)
-          if (mq[s] <= thr.v[s] * thr.m[s]) hitm |= 1u << s;
+          if (mq[s] <= thr.vm[s]) hitm |= 1u << s;
       }
       cE = mE;
       cT = mT;
@@ -491,9 +485,8 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
       par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
     if (hit || par) {
-      thr_to_sm<WS>(thr, thr_sm);
       nref += tile_slow<WS>(tb, p, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
-      thr_from_sm<WS>(thr, thr_sm);
+      thr_from_sm<WS>(p, thr, thr_sm);
     }
   }
   __syncwarp();
@@ -520,12 +513,8 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   BestRec lb[WS::N > 0 ? WS::N : 1];
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {
-    if constexpr (WS::RT) {
-      thr_sm[s] = __int_as_float(0x7f800000);
-    } else {
-      thr.v[s] = __int_as_float(0x7f800000);
-      thr.m[s] = s < WS::N ? p.mul[p.ws_perm[s]] : 1.f;
-    }
+    thr_sm[s] = __int_as_float(0x7f800000);
+    if constexpr (!WS::RT) thr.vm[s] = __int_as_float(0x7f800000);
     best_init(lb[s]);
   }
   const int nws = WS::RT ? p.nw : WS::N;  // weights searched
@@ -550,12 +539,12 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     s = s > p.lo ? s : p.lo;
     e = e < p.hi ? e : p.hi;
     if (s >= e) continue;
-    if constexpr (WS::RT) {
-      for (int w = 0; w < nws; w++) thr_sm[w] = fminf(thr_sm[w], __uint_as_float(__ldcg(p.thr + w)));
-    } else {
 #pragma unroll
-      for (int w = 0; w < WS::N; w++) thr.v[w] = fminf(thr.v[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
+    for (int w = 0; w < WS::N; w++) {
+      if (w >= nws) break;
+      thr_sm[w] = fminf(thr_sm[w], __uint_as_float(__ldcg(p.thr + p.ws_perm[w])));
     }
+    thr_from_sm<WS>(p, thr, thr_sm);
     if (p.want_pareto) {
       u64 sv = wp.sver;
       stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
@@ -612,11 +601,10 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
 #pragma unroll
     for (int w = 0; w < WS::N; w++) {
       if (w >= nws) break;
-      float t = WS::RT ? thr_sm[w] : thr.v[w];
+      float t = thr_sm[w];
 #pragma unroll
       for (int o = 16; o; o >>= 1) t = fminf(t, __shfl_xor_sync(0xffffffffu, t, o));
-      if constexpr (WS::RT) thr_sm[w] = t;
-      else thr.v[w] = t;
+      thr_sm[w] = t;
       if (lane == 0 && t < __uint_as_float(__ldcg(p.thr + p.ws_perm[w])))
         atomicMin(p.thr + p.ws_perm[w], __float_as_uint(t));
     }
