@@ -84,7 +84,7 @@ def test_ctile2_equals_path5_on_a_c3client_slice(monkeypatch):
     group-table kernel equals the per-client tile kernel (path 5) bitwise,
     and its picks re-score bitwise in the oracle."""
     prof, q = c3client()
-    lo = 1000 << 24
+    lo = 5000 << 24   # 64 feasible partitions (partitions 1000..1063 are all memory-infeasible)
     qw = q.with_range(lo, lo + (1 << 30))
     sch = S.Scheduler(prof)
     r6 = sch.search(qw)
@@ -96,6 +96,7 @@ def test_ctile2_equals_path5_on_a_c3client_slice(monkeypatch):
     assert [(p.index, p.makespan_s, p.energy_j) for p in r6.pareto] == \
         [(p.index, p.makespan_s, p.energy_j) for p in r5.pareto]
     assert r6.stats["n_configs"] == r5.stats["n_configs"] == 1 << 30
+    assert r6.stats["n_feasible"] > 0 and all(b.valid for b in r6.best)
     for p in list(r6.pareto) + list(r6.best):
         ok, T, E = oracle.score(prof, q, *oracle.config(q, p.index))
         assert ok and (T, E) == (p.makespan_s, p.energy_j)

@@ -92,3 +92,17 @@ def test_client_certificate_parallel_equals_serial():
     a = oracle.dp_certificate(prof, q)
     b = oracle.dp_certificate(prof, q, procs=3)
     assert a["front"] == b["front"] and a["best"] == b["best"]
+
+
+@pytest.mark.parametrize("n,g,c,seed", [(9, 5, 9, 730), (10, 4, 4, 731), (10, 8, 3, 732)])
+def test_client_certificate_equals_enumeration_n9_n10(n, g, c, seed):
+    """O4 == O1 (full enumeration, process pool) at the largest PER_CLIENT
+    sizes the enumerator covers in seconds: n = 9, 10 with 2 levels per
+    client (pin O4 beyond n = 8 before trusting it at n = 16)."""
+    from synth import PER_CLIENT
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, (50, 100), PER_CLIENT, W, True)
+    r = oracle.search_parallel(prof, q)
+    cert = oracle.dp_certificate(prof, q, procs=2)
+    assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
+    assert [b[1] if b else None for b in r["best"]] == cert["best"]
