@@ -124,7 +124,8 @@ enum {
   kCtrFront = 7,     // finalize: front size
   kCtrStairVer = 8,  // staircase version (bumped per insertion)
   kCtrPass = 9,      // search passes run
-  kCtrN = 16
+  kCtrB0 = 16,       // [kMaxW] best exact F64 (bits, atomicMax) recorded so far, weights with b = 0
+  kCtrN = 24
 };
 
 struct BestRec {      // 48 B

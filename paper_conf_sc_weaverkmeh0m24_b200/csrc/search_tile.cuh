@@ -169,6 +169,30 @@ __device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec 
   return out;
 }
 
+// bit s set: weight s has b = 0 and F(T64) = X^a is STRICTLY below the best
+// exact F recorded by any lane so far (ctr[kCtrB0 + w]): every configuration
+// with makespan >= T64 is strictly worse than a real configuration, whatever
+// its index
+template <class WS>
+__device__ __forceinline__ unsigned b0_below_global(const DevParams &p, unsigned mask, double T64) {
+  unsigned out = 0;
+  if constexpr (WS::RT) {
+    for (int s = 0; s < p.nw; s++)
+      if ((mask >> s & 1u) && p.wb[s] == 0) {
+        const double Fg = __longlong_as_double((long long)__ldcg(p.ctr + kCtrB0 + s));
+        if (Fg > 0.0 && objective64(p, T64, 1.0, p.wa[s], 0) < Fg) out |= 1u << s;
+      }
+  } else {
+#pragma unroll
+    for (int s = 0; s < WS::N; s++)
+      if (WS::B(s) == 0 && (mask >> s & 1u)) {
+        const double Fg = __longlong_as_double((long long)__ldcg(p.ctr + kCtrB0 + p.ws_perm[s]));
+        if (Fg > 0.0 && objective64(p, T64, 1.0, WS::A(s), 0) < Fg) out |= 1u << s;
+      }
+  }
+  return out;
+}
+
 // mask of the weights with b = 0
 template <class WS>
 __device__ __forceinline__ unsigned b0_mask(const DevParams &p) {
@@ -227,6 +251,7 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
   // the lane's best (b0_beaten) -- stops the tie flood of (1,0), where every
   // configuration sharing the optimum's bottleneck group ties it
   need &= ~b0_beaten<WS>(p, lb, need, T64, idx);
+  need &= ~b0_below_global<WS>(p, need, T64);
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
   // fp64 canonical re-score from the exact group tuples: T = max_g T_g (exact),
@@ -249,6 +274,8 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
           b.t32 = T;
           b.e32 = E;
           b.valid = 1;
+          if ((WS::RT ? p.wb[s] : WS::B(s)) == 0)   // publish: every lane may drop worse F (b0_below_global)
+            atomicMax(p.ctr + kCtrB0 + p.ws_perm[s], (unsigned long long)__double_as_longlong(F));
         }
       }
     }
@@ -405,7 +432,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
       double pc = 0.0;
       for (int b = 0; b < k; b++)
         pc = fmax(pc, fmin(fmin(wp.g64[b * 4], wp.g64[b * 4 + 1]), fmin(wp.g64[b * 4 + 2], wp.g64[b * 4 + 3])));
-      b0skip = b0_beaten<WS>(p, lb, b0m, pc, wp.base + v0);
+      b0skip = b0_beaten<WS>(p, lb, b0m, pc, wp.base + v0) | b0_below_global<WS>(p, b0m, pc);
     }
   }
   const float minTin = WS::N > 0 ? 0.f
@@ -478,7 +505,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
     if (hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
       c64 = tile_corner64(wp, vt);
-      hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+      hitm &= ~(b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt) | b0_below_global<WS>(p, hitm, c64));
     }
     const bool hit = hitm != 0;
     bool par = false;
