@@ -38,6 +38,8 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
     dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
     dp.unit_stride = 1;
   }
+  err = publish_params(dp, st);
+  if (err != cudaSuccess) return err;
   void *args[] = {(void *)&dp};
   cudaEventRecord(e1, st);
   err = cudaLaunchKernel(tl.fn, *grid, kC2Threads, args, tl.smem, st);

@@ -111,6 +111,11 @@ struct DevParams {
   unsigned char *out;          // finalize output area
   const unsigned char *gtab;   // [2^n][L] GroupRec: fp32/fp64 group tuples (nullptr: compute)
   int gtab_ok;                 // workspace holds a group table for this query
+  int b0mode;                  // tile kernel, weights with b = 0: bit 0 partition-level, bit 1 tile-level
+                               // early reject (default 3; SCHED_B0 overrides, measurement only)
+  const DevParams *gp;         // this block's copy in the workspace (global memory): handed to the
+                               // out-of-line slow paths, so no thread copies the kernel parameters
+                               // to its stack (local memory)
 };
 
 enum {
@@ -124,8 +129,7 @@ enum {
   kCtrFront = 7,     // finalize: front size
   kCtrStairVer = 8,  // staircase version (bumped per insertion)
   kCtrPass = 9,      // search passes run
-  kCtrB0 = 16,       // [kMaxW] best exact F64 (bits, atomicMax) recorded so far, weights with b = 0
-  kCtrN = 24
+  kCtrN = 16
 };
 
 struct BestRec {      // 48 B

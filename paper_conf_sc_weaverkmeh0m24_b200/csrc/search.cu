@@ -495,7 +495,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, fin, out, gtab, total;
+  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, fin, out, gtab, params, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -518,6 +518,7 @@ WsLayout layout(const DevParams &dp) {
   L.cand = take(sizeof(CandRec) * (size_t)dp.cand_cap);
   L.surv = take(4 * (size_t)dp.cand_cap);
   L.fin = take(finalize_bytes(dp.cand_cap));
+  L.params = take(sizeof(DevParams));
   L.out = take(sizeof(BestRec) * kMaxW + sizeof(CandRec) * (size_t)kFrontCap);
   L.gtab = take(dp.gtab_ok ? sizeof(GroupRec) * ((size_t)dp.L << dp.n) : 0);
   L.total = (o + 255) / 256 * 256;
@@ -612,6 +613,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.cand = ws + L.cand;
   dp.out = ws + L.out;
   dp.gtab = dp.gtab_ok ? ws + L.gtab : nullptr;
+  dp.gp = (const DevParams *)(ws + L.params);
   int dev = 0, nsm = 0;
   CK(cudaGetDevice(&dev));
   CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));
@@ -727,6 +729,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
       CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_generic, kThreads, smem));
       if (occ < 1) return SCHED_E_TOO_LARGE;
       grid = std::min(kMaxGrid, nsm * occ);
+      CK(publish_params(dp, st));
       CK(cudaEventRecord(e1, st));
       k_generic<<<grid, kThreads, smem, st>>>(dp);
       CK(cudaGetLastError());

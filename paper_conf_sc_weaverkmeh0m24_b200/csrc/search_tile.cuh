@@ -169,30 +169,6 @@ __device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec 
   return out;
 }
 
-// bit s set: weight s has b = 0 and F(T64) = X^a is STRICTLY below the best
-// exact F recorded by any lane so far (ctr[kCtrB0 + w]): every configuration
-// with makespan >= T64 is strictly worse than a real configuration, whatever
-// its index
-template <class WS>
-__device__ __forceinline__ unsigned b0_below_global(const DevParams &p, unsigned mask, double T64) {
-  unsigned out = 0;
-  if constexpr (WS::RT) {
-    for (int s = 0; s < p.nw; s++)
-      if ((mask >> s & 1u) && p.wb[s] == 0) {
-        const double Fg = __longlong_as_double((long long)__ldcg(p.ctr + kCtrB0 + s));
-        if (Fg > 0.0 && objective64(p, T64, 1.0, p.wa[s], 0) < Fg) out |= 1u << s;
-      }
-  } else {
-#pragma unroll
-    for (int s = 0; s < WS::N; s++)
-      if (WS::B(s) == 0 && (mask >> s & 1u)) {
-        const double Fg = __longlong_as_double((long long)__ldcg(p.ctr + kCtrB0 + p.ws_perm[s]));
-        if (Fg > 0.0 && objective64(p, T64, 1.0, WS::A(s), 0) < Fg) out |= 1u << s;
-      }
-  }
-  return out;
-}
-
 // mask of the weights with b = 0
 template <class WS>
 __device__ __forceinline__ unsigned b0_mask(const DevParams &p) {
@@ -251,7 +227,6 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
   // the lane's best (b0_beaten) -- stops the tie flood of (1,0), where every
   // configuration sharing the optimum's bottleneck group ties it
   need &= ~b0_beaten<WS>(p, lb, need, T64, idx);
-  need &= ~b0_below_global<WS>(p, need, T64);
   const bool par = p.want_pareto && !stair_dominated(stair, p, T64, E);
   if (!need && !par) return 0;
   // fp64 canonical re-score from the exact group tuples: T = max_g T_g (exact),
@@ -274,8 +249,6 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
           b.t32 = T;
           b.e32 = E;
           b.valid = 1;
-          if ((WS::RT ? p.wb[s] : WS::B(s)) == 0)   // publish: every lane may drop worse F (b0_below_global)
-            atomicMax(p.ctr + kCtrB0 + p.ws_perm[s], (unsigned long long)__double_as_longlong(F));
         }
       }
     }
@@ -390,7 +363,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                                  uint32_t v0, uint32_t v1, int lane) {
   const int k = wp.cfg.k;
   if (k < 5) {
-    const int r = edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
+    const int r = edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
     thr_from_sm<WS>(p, thr, thr_sm);
     return r;
   }
@@ -427,12 +400,12 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
   // it) never reaches the per-tile exact corner
   unsigned b0skip = 0;
   {
-    const unsigned b0m = b0_mask<WS>(p);
+    const unsigned b0m = (p.b0mode & 1) ? b0_mask<WS>(p) : 0u;
     if (b0m) {
       double pc = 0.0;
       for (int b = 0; b < k; b++)
         pc = fmax(pc, fmin(fmin(wp.g64[b * 4], wp.g64[b * 4 + 1]), fmin(wp.g64[b * 4 + 2], wp.g64[b * 4 + 3])));
-      b0skip = b0_beaten<WS>(p, lb, b0m, pc, wp.base + v0) | b0_below_global<WS>(p, b0m, pc);
+      b0skip = b0_beaten<WS>(p, lb, b0m, pc, wp.base + v0);
     }
   }
   const float minTin = WS::N > 0 ? 0.f
@@ -448,7 +421,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     const float2 lp = wp.lp[j];
     const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
     if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-      nref += edge_configs<WS>(tb, p, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+      nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
       thr_from_sm<WS>(p, thr, thr_sm);
       continue;
     }
@@ -503,16 +476,16 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     }
     hitm &= ~b0skip;
     double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
-    if (hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
+    if ((p.b0mode & 2) && hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
       c64 = tile_corner64(wp, vt);
-      hitm &= ~(b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt) | b0_below_global<WS>(p, hitm, c64));
+      hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
     }
     const bool hit = hitm != 0;
     bool par = false;
     if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
       par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
     if (hit || par) {
-      nref += tile_slow<WS>(tb, p, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+      nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
       thr_from_sm<WS>(p, thr, thr_sm);
     }
   }
@@ -574,12 +547,12 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     thr_from_sm<WS>(p, thr, thr_sm);
     if (p.want_pareto) {
       u64 sv = wp.sver;
-      stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
+      stair_sync(stair, *p.gp, sv, __ldcg(p.ctr + kCtrStairVer));
       __syncwarp();
       if (lane == 0) wp.sver = sv;
     }
     if (lane == 0) {
-      dev_unrank(tb, p, s, wp.cfg);
+      dev_unrank(tb, *p.gp, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
@@ -587,7 +560,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     for (;;) {
       if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
         u64 sv = wp.sver;
-        stair_sync(stair, p, sv, ver_pref);
+        stair_sync(stair, *p.gp, sv, ver_pref);
         ver_pref = __ldcg(p.ctr + kCtrStairVer);  // consumed next partition: load latency off the path
         __syncwarp();
         if (lane == 0) wp.sver = sv;
@@ -619,7 +592,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
       if (base + Pn >= e) break;
       if (lane == 0) {
         wp.base = base + Pn;
-        dev_successor(tb, p, wp.cfg);
+        dev_successor(tb, *p.gp, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
       }

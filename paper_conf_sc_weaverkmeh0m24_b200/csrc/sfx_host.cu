@@ -41,6 +41,8 @@ cudaError_t launch_sfx(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_
     dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
     dp.unit_stride = 1;
   }
+  err = publish_params(dp, st);
+  if (err != cudaSuccess) return err;
   void *args[] = {(void *)&dp};
   cudaEventRecord(e1, st);
   err = cudaLaunchKernel(tl.fn, *grid, kSfxThreads, args, tl.smem, st);

@@ -57,6 +57,8 @@ size_t tile_smem_bytes(const DevParams &dp) {
 }
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
+  const char *b0 = std::getenv("SCHED_B0");
+  dp.b0mode = b0 && *b0 ? std::atoi(b0) : 3;
   if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4 || !dp.gtab_ok) return false;
   // E = sum_g E_g with level-independent feasibility: COUNT_IDLE (global
   // energy term) and NO_INTERFERENCE (level-dependent feasibility) take the generic kernel
@@ -87,6 +89,8 @@ cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream
     dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
     dp.unit_stride = 1;
   }
+  err = publish_params(dp, st);
+  if (err != cudaSuccess) return err;
   void *args[] = {(void *)&dp};
   cudaEventRecord(e1, st);
   err = cudaLaunchKernel(tl.fn, *grid, kTileThreads, args, tl.smem, st);

@@ -39,6 +39,10 @@ constexpr int kTileWarps = kTileThreads / 32;
 constexpr int kTileMaxL = 4;
 constexpr int kTileMaxG = 8;
 size_t tile_smem_bytes(const DevParams &dp);
+// the launch's DevParams -> its workspace copy (dp.gp), before the kernel
+inline cudaError_t publish_params(const DevParams &dp, cudaStream_t st) {
+  return cudaMemcpyAsync((void *)dp.gp, &dp, sizeof dp, cudaMemcpyHostToDevice, st);
+}
 bool tile_eligible(DevParams &dp, TileLaunch *tl);
 bool dfs_eligible(DevParams &dp, TileLaunch *tl);
 bool sfx_eligible(DevParams &dp, TileLaunch *tl);
