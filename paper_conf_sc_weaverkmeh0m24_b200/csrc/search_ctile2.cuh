@@ -281,14 +281,14 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
     for (int w = 0; w < WM; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
     if (lane == 0) {
-      dev_unrank(tb, p, s, wp.cfg);
+      dev_unrank(tb, *p.gp, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
     for (;;) {
       if (p.want_pareto) {
         u64 sv = wp.sver;
-        stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
+        stair_sync(stair, *p.gp, sv, __ldcg(p.ctr + kCtrStairVer));
         __syncwarp();
         if (lane == 0) wp.sver = sv;
       }
@@ -307,7 +307,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
         uint32_t voL, tbits;
         c2_tables(tb, p, wp, lane);
         if (k < 3) {
-          nref += c2_small<WM>(tb, p, stair, wp, thr, lb, v0, v1, lane);
+          nref += c2_small<WM>(tb, *p.gp, stair, wp, thr, lb, v0, v1, lane);
         } else {
           c2_setup(p, wp, lane, idxL, voL, tbits);
           const uint32_t nout = 1u << (2 * (n - 3));
@@ -403,7 +403,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
               const bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(mT, p.tlb_scale_f), mE);
               if (!hit && !par) continue;
             }
-            nref += c2_tile_slow<WM>(tb, p, stair, wp, thr, lb, o, vo, v0, v1, Tp, Ep, At, Ae, Bt, Be, Ct, Ce);
+            nref += c2_tile_slow<WM>(tb, *p.gp, stair, wp, thr, lb, o, vo, v0, v1, Tp, Ep, At, Ae, Bt, Be, Ct, Ce);
           }
         }
       }
@@ -411,10 +411,10 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
       if (base + Pn >= e) break;
       if (lane == 0) {
         wp.base = base + Pn;
-        dev_successor(tb, p, wp.cfg);
+        dev_successor(tb, *p.gp, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
-        cfg_feasibility(tb, p, wp.cfg);
+        cfg_feasibility(tb, *p.gp, wp.cfg);
       }
       __syncwarp();
     }

@@ -58,7 +58,7 @@ size_t tile_smem_bytes(const DevParams &dp) {
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
   const char *b0 = std::getenv("SCHED_B0");
-  dp.b0mode = b0 && *b0 ? std::atoi(b0) : 3;
+  dp.b0mode = b0 && *b0 ? std::atoi(b0) : 2;  // tile-level only: the partition-level pass costs more than it saves (c4 (1,0): 740 vs 779 ms)
   if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4 || !dp.gtab_ok) return false;
   // E = sum_g E_g with level-independent feasibility: COUNT_IDLE (global
   // energy term) and NO_INTERFERENCE (level-dependent feasibility) take the generic kernel
