@@ -86,13 +86,15 @@ def test_dp_front_c4_literal_per_client():
           [b.score64 for b in best], "vs per-GPU", [b.score64 for b in bg])
 
 
-@pytest.mark.parametrize("n", [13, 14])
+@pytest.mark.parametrize("n", [13, 14, 16])
 def test_dp_front_c4_client_prefix_golden(n):
-    """Literal per-client reading on the c4 profile at the largest sizes the
-    O4 oracle runs (the first 13 / 14 workflows, G = 8, 4 levels per client:
-    5.9e13 / 7.3e14+ configurations): front values and optimum per weight
-    bitwise equal to the stored certificate (tests/golden, written by
-    `python -m oracle.make_certificates client n`)."""
+    """Literal per-client reading on the c4 profile: the first 13 / 14
+    workflows and the whole c4 queue (n = 16: 4.05e19 configurations, the
+    north star's "per-client active-thread percentage"), G = 8, 4
+    levels per client: front values and optimum per weight bitwise equal to
+    the stored O4 certificate (tests/golden, written by
+    `python -m oracle.make_certificates client n [procs]`; n = 16 took 75
+    minutes on 7 host processes)."""
     import json
     import os
     g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", f"c4_client_n{n}_certificate.json")))

@@ -106,3 +106,28 @@ def test_client_certificate_equals_enumeration_n9_n10(n, g, c, seed):
     cert = oracle.dp_certificate(prof, q, procs=2)
     assert [(t, e) for _, t, e in r["pareto"]] == cert["front"]
     assert [b[1] if b else None for b in r["best"]] == cert["best"]
+
+
+def test_client_n16_certificate_consistent_with_per_gpu_certificate():
+    """The literal per-client c4 certificate (O4, n = 16) against the PER_GPU
+    c4 certificate (O3), two independent computations: every PER_GPU
+    configuration is also a PER_CLIENT configuration (all clients of a group
+    at the group's level), so every PER_GPU front point is weakly dominated
+    by a per-client front point and every per-client optimum is >= the
+    PER_GPU one.  Also: the stored baselines equal the oracle's constants."""
+    g16 = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c4_client_n16_certificate.json")))
+    g4 = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "c4_certificate.json")))
+    f16 = [(float.fromhex(t), float.fromhex(e)) for t, e in g16["front_T_E"]]
+    f4 = [(float.fromhex(t), float.fromhex(e)) for t, e in g4["front_T_E"]]
+    assert f16 == sorted(f16) and all(a[1] > b[1] for a, b in zip(f16, f16[1:]))   # a staircase
+    for t, e in f4:
+        assert any(t2 <= t and e2 <= e for t2, e2 in f16)
+    w16 = [tuple(w) for w in g16["weights"]]
+    for w, b in zip(g4["weights"], g4["best_score64"]):
+        assert float.fromhex(g16["best_score64"][w16.index(tuple(w))]) >= float.fromhex(b)
+    prof, q = config("c4")
+    ts, es = oracle.constants(prof, q)
+    assert g16["tseq"] == ts.hex() and g16["eseq"] == es.hex()
+    # the optimum of each weight is attained on the stored front
+    for (a, b), best in zip(w16, g16["best_score64"]):
+        assert max(oracle.objective(ts, es, t, e, a, b) for t, e in f16) == float.fromhex(best)
