@@ -239,6 +239,30 @@ def run_dry(args):
     return 0
 
 
+def secondary(S):
+    """The other kernels on their BASELINE workloads, one device-timed search
+    each after a warm-up (context for the headline, not the headline):
+    the literal per-client c3 ("c3-client", 1/64 chunk slice; kernel_path 6)
+    and the whole c5 space (7-weight sweep + Pareto; kernel_path 3)."""
+    from synth import config, Query
+    out = []
+    prof3, q3 = config("c3")
+    qc = Query(q3.n, q3.g, q3.c, q3.levels, 0, q3.weights, q3.want_pareto)
+    prof5, q5 = config("c5")
+    for name, prof, q, kw in (("c3-client (PER_CLIENT c3, 5.5e13 configs), 1/64 slice", prof3, qc,
+                               {"shard": (5, 64), "chunk_log2": CHUNK_LOG2}),
+                              ("c5 whole space (7-weight sweep + Pareto)", prof5, q5, {})):
+        sch = S.Scheduler(prof)
+        sch.search(q, **kw)
+        r = sch.search(q, **kw)
+        st = r.stats
+        out.append({"workload": name, "configs": st["n_configs"], "search_ms": st["search_ms"],
+                    "configs_per_s": st["n_configs"] / (st["search_ms"] / 1e3), "kernel_path": st["kernel_path"],
+                    "feasible_fraction": st["n_feasible"] / max(1, st["n_configs"])})
+        sch.close()
+    return out
+
+
 def describe(name, q):
     """The workload's one-line description (BASELINE.json configs, synth/configs.py)."""
     idx = {"c1": 0, "c2": 1, "c3": 2, "c4": 3, "c5": 4}.get(name)
@@ -420,6 +444,8 @@ def run_ours(args):
                              f"peak = {SMS} SMs x 4 SMSP x 32 lanes x {f_max:.0f} MHz (sm_max_mhz, "
                              "MEASURED_PEAKS.json) issue slots"},
     }
+    if world == 1 and not args.no_secondary:
+        line["config"]["secondary"] = secondary(S)
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(prof, q)
     print(json.dumps(line), flush=True)
@@ -462,6 +488,7 @@ def main():
     ap.add_argument("--workload", default="c4")
     ap.add_argument("--full", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true")
     ap.add_argument("--ref-window", type=int, default=400_000)
     ap.add_argument("--dry-run", action="store_true", help="CPU/gloo plumbing test, no kernels")
     args = ap.parse_args()

@@ -253,14 +253,14 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
 #pragma unroll
     for (int w = 0; w < WM; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
-    if (p.want_pareto) stair_sync(stair, *p.gp, stair_ver, __ldcg(p.ctr + kCtrStairVer));
+    if (p.want_pareto) stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     if (lane == 0) {
-      dev_unrank(tb, *p.gp, s, wp.cfg);
+      dev_unrank(tb, p, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
     for (;;) {
-      if (p.want_pareto) stair_sync(stair, *p.gp, stair_ver, __ldcg(p.ctr + kCtrStairVer));
+      if (p.want_pareto) stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
       const u64 base = wp.base;
       const uint32_t Pn = (uint32_t)wp.cfg.Pn;
       const int k = wp.cfg.k;
@@ -377,10 +377,10 @@ __global__ void __launch_bounds__(kCtThreads, 2) k_ctile(const DevParams p) {
       if (base + Pn >= e) break;
       if (lane == 0) {
         wp.base = base + Pn;
-        dev_successor(tb, *p.gp, wp.cfg);
+        dev_successor(tb, p, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
-        cfg_feasibility(tb, *p.gp, wp.cfg);
+        cfg_feasibility(tb, p, wp.cfg);
       }
       __syncwarp();
     }

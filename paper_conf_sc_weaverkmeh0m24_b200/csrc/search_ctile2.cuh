@@ -281,14 +281,14 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
     for (int w = 0; w < WM; w++)
       if (w < p.nw) thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
     if (lane == 0) {
-      dev_unrank(tb, *p.gp, s, wp.cfg);
+      dev_unrank(tb, p, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
     for (;;) {
       if (p.want_pareto) {
         u64 sv = wp.sver;
-        stair_sync(stair, *p.gp, sv, __ldcg(p.ctr + kCtrStairVer));
+        stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
         __syncwarp();
         if (lane == 0) wp.sver = sv;
       }
@@ -411,10 +411,10 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
       if (base + Pn >= e) break;
       if (lane == 0) {
         wp.base = base + Pn;
-        dev_successor(tb, *p.gp, wp.cfg);
+        dev_successor(tb, p, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
-        cfg_feasibility(tb, *p.gp, wp.cfg);
+        cfg_feasibility(tb, p, wp.cfg);
       }
       __syncwarp();
     }

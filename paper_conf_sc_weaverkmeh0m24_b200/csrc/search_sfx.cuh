@@ -518,16 +518,16 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
 #pragma unroll
     for (int q = 0; q < kMaxW; q++)
       if (q < p.nw) cold.thr[q] = fminf(cold.thr[q], __uint_as_float(__ldcg(p.thr + q)));
-    if (p.want_pareto) stair_sync(stair, *p.gp, stair_ver, __ldcg(p.ctr + kCtrStairVer));
+    if (p.want_pareto) stair_sync(stair, p, stair_ver, __ldcg(p.ctr + kCtrStairVer));
     if (lane == 0) {
-      const uint32_t r = sfx_unrank_prefix(tb, *p.gp, s, w.cfg, plen);
+      const uint32_t r = sfx_unrank_prefix(tb, p, s, w.cfg, plen);
       w.base = s - r;
     }
     __syncwarp();
     u64 ver_pref = p.want_pareto ? __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0) : 0;
     for (;;) {
       if (p.want_pareto) {
-        stair_sync(stair, *p.gp, stair_ver, ver_pref);
+        stair_sync(stair, p, stair_ver, ver_pref);
         ver_pref = __shfl_sync(0xffffffffu, __ldcg(p.ctr + kCtrStairVer), 0);
       }
       const int kp = w.cfg.k;
@@ -613,7 +613,7 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
       if (base + Wp >= e) break;
       if (lane == 0) {
         w.base = base + Wp;
-        w.flag = sfx_prefix_successor(tb, *p.gp, w.cfg, plen - 1) ? 1 : 0;
+        w.flag = sfx_prefix_successor(tb, p, w.cfg, plen - 1) ? 1 : 0;
       }
       __syncwarp();
       if (!w.flag) break;

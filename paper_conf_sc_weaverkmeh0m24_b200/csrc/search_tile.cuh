@@ -414,17 +414,23 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                          fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
   int nref = 0;
   const uint32_t s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
+  // Every rare path of the tile loop (unit-boundary tiles, exact corners,
+  // slow re-checks) is entered warp-uniformly (a vote), so the common
+  // iteration carries no convergence-barrier bookkeeping; lanes without work
+  // in a rare path skip it inside.
   for (uint32_t st = s_lo; st <= s_hi; st++) {
     const uint32_t j = 2 * st + h;
     const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
-    if (j >= (uint32_t)nloop || vt + 64 <= v0 || vt >= v1) continue;
-    const float2 lp = wp.lp[j];
-    const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
-    if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-      nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+    const bool live = j < (uint32_t)nloop && vt + 64 > v0 && vt < v1;
+    const bool part = live && (vt < v0 || vt + 64 > v1);
+    if (__any_sync(0xffffffffu, part)) {  // partial tiles at a unit boundary
+      if (part)
+        nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
       thr_from_sm<WS>(p, thr, thr_sm);
-      continue;
     }
+    const bool full = live && !part;
+    const float2 lp = wp.lp[j < (uint32_t)nloop ? j : 0u];
+    const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
     unsigned hitm = 0;
     float cE, cT;
     if constexpr (WS::N > 0) {
@@ -474,18 +480,24 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         }
       }
     }
-    hitm &= ~b0skip;
-    double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
-    if ((p.b0mode & 2) && hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
-      c64 = tile_corner64(wp, vt);
-      hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+    hitm = full ? (hitm & ~b0skip) : 0u;
+    // exact tile corner (fp64 min makespan) where a screen needs it: b = 0
+    // weights (no configuration of the tile beats the lane's best) and the
+    // Pareto screen when the fp32 staircase test cannot decide
+    const bool b0c = (p.b0mode & 2) && hitm && b0_any<WS>(p, hitm);
+    const bool fpar = full && p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE);
+    bool par = false;
+    if (__any_sync(0xffffffffu, b0c || fpar)) {
+      if (b0c || fpar) {
+        const double c64 = tile_corner64(wp, vt);
+        if (b0c) hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+        if (fpar) par = !stair_dominated(stair, p, c64, cE);
+      }
     }
     const bool hit = hitm != 0;
-    bool par = false;
-    if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
-      par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
-    if (hit || par) {
-      nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+    const bool slow = hit || par;
+    if (__any_sync(0xffffffffu, slow)) {
+      if (slow) nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
       thr_from_sm<WS>(p, thr, thr_sm);
     }
   }
@@ -547,12 +559,12 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     thr_from_sm<WS>(p, thr, thr_sm);
     if (p.want_pareto) {
       u64 sv = wp.sver;
-      stair_sync(stair, *p.gp, sv, __ldcg(p.ctr + kCtrStairVer));
+      stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
       __syncwarp();
       if (lane == 0) wp.sver = sv;
     }
     if (lane == 0) {
-      dev_unrank(tb, *p.gp, s, wp.cfg);
+      dev_unrank(tb, p, s, wp.cfg);
       wp.base = s - wp.cfg.v;
     }
     __syncwarp();
@@ -560,7 +572,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
     for (;;) {
       if (p.want_pareto) {  // staircase refresh per partition (version prefetched one partition ahead)
         u64 sv = wp.sver;
-        stair_sync(stair, *p.gp, sv, ver_pref);
+        stair_sync(stair, p, sv, ver_pref);
         ver_pref = __ldcg(p.ctr + kCtrStairVer);  // consumed next partition: load latency off the path
         __syncwarp();
         if (lane == 0) wp.sver = sv;
@@ -592,7 +604,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
       if (base + Pn >= e) break;
       if (lane == 0) {
         wp.base = base + Pn;
-        dev_successor(tb, *p.gp, wp.cfg);
+        dev_successor(tb, p, wp.cfg);
         wp.cfg.Pn = tb.W[wp.cfg.st[p.n - 1]];
         wp.cfg.v = 0;
       }
