@@ -418,7 +418,7 @@ def run_ours(args):
     achieved = OPS_PER_CONFIG * ncfg / (search_ms / 1e3) / 1e12
     traffic = None
     try:
-        prof_sum = json.load(open(os.path.join(ROOT, "profiles", "r01_traffic.json")))
+        prof_sum = json.load(open(os.path.join(ROOT, "profiles", "r02_traffic.json")))
         traffic = prof_sum["dram_bytes_per_config"] * (ncfg / args.steps)
     except Exception:
         pass

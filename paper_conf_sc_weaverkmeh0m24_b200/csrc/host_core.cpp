@@ -559,6 +559,15 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
     const double eta = q.wa[w] * eT + q.wb[w] * eE + (q.wa[w] + q.wb[w] + 2.0) * u;
     dp->delta[w] = (float)(4.0 * eta);
     dp->mul[w] = 1.f + dp->delta[w];
+    // log-domain pre-screen of the run-time-weight tile kernel (search_tile.cuh
+    // rt_screen): a*lg2(T) + b*lg2(E) <= lg2(thr * mul) + lmargin whenever the
+    // exact proxy test passes, for |lg2| <= 32 of every operand: each __log2f
+    // is within 2^-17 absolute there (2 ulp relative), the fp32 proxy within
+    // (a+b) u of T^a E^b, the FMUL/FFMA within |L| 2^-23 -- (a+b+1) 2^-15
+    // covers the sum with room
+    dp->fa[w] = (float)q.wa[w];
+    dp->fb[w] = (float)q.wb[w];
+    dp->lmargin[w] = (float)std::ldexp((double)(q.wa[w] + q.wb[w] + 1), -15);
   }
   dp->gamma = (float)(2.0 * std::max(eT, eE) + 4.0 * u);
   dp->tlb_scale = std::nextafter(tseq / (1.0 + 2.0 * eT), 0.0);

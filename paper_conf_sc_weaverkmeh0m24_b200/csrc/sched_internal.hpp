@@ -74,6 +74,8 @@ struct DevParams {
   float gamma;              // Pareto "surely dominated" margin
   int ws_perm[kMaxW];       // tile kernel: compile-time weight slot -> query weight index
   float mul[kMaxW];         // 1 + delta[w]
+  float fa[kMaxW], fb[kMaxW];  // the exponents as floats (run-time-weight tile screen, log domain)
+  float lmargin[kMaxW];     // its conservative margin in log2 units (host_core.cpp)
   double tlb_scale;         // T_seq / (1 + 2 eps_T) rounded down: T64 >= T32hat * tlb_scale
   float tlb_scale_f;        // the same, as a float rounded down
   float phat;               // P_s * T_seq / E_seq

@@ -169,6 +169,18 @@ __device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec 
   return out;
 }
 
+// does the (compile-time) weight set contain a b = 0 weight? (run-time sets: maybe)
+template <class WS>
+__host__ __device__ constexpr bool ws_has_b0() {
+  if constexpr (WS::RT) {
+    return true;
+  } else {
+    for (int s = 0; s < WS::N; s++)
+      if (WS::B(s) == 0) return true;
+    return false;
+  }
+}
+
 // mask of the weights with b = 0
 template <class WS>
 __device__ __forceinline__ unsigned b0_mask(const DevParams &p) {
@@ -350,7 +362,33 @@ __device__ __forceinline__ void thr_from_sm(const DevParams &p, Thr<WS> &thr, co
   if constexpr (!WS::RT) {
 #pragma unroll
     for (int s = 0; s < WS::N; s++) thr.vm[s] = thr_sm[s] * p.mul[p.ws_perm[s]];
+  } else {  // log2 thresholds of the pre-screen (rt_screen), +inf while unset
+#pragma unroll
+    for (int s = 0; s < kMaxW; s++)
+      if (s < p.nw) thr.vm[s] = __log2f(thr_sm[s] * p.mul[s]) + p.lmargin[s];
   }
+}
+
+// run-time-weight corner screen: bit s set iff q_s(mT, mE) <= thr_s (1 + delta_s).
+// A log-domain pre-screen (2 MUFU per tile, 2 FMA-pipe ops + 1 compare per
+// weight, exponents from the constant bank) is passed by every weight that
+// the exact test passes (lmargin, host_core.cpp); only those run the exact
+// repeated-multiplication test.  Operands outside 2^+-32 skip the pre-screen.
+template <class WS>
+__device__ __forceinline__ unsigned rt_screen(const DevParams &p, const Thr<WS> &thr, const float *thr_sm, float mT,
+                                              float mE) {
+  const float lt = __log2f(mT), le = __log2f(mE);
+  const bool inr = fabsf(lt) < 32.f && fabsf(le) < 32.f;
+  unsigned pre = 0;
+#pragma unroll
+  for (int s = 0; s < kMaxW; s++)
+    if (s < p.nw && (!inr || fmaf(p.fa[s], lt, p.fb[s] * le) <= thr.vm[s])) pre |= 1u << s;
+  unsigned hit = 0;
+  if (pre) {
+    for (int s = 0; s < p.nw; s++)
+      if ((pre >> s & 1u) && rt_q(p, s, mT, mE) <= thr_sm[s] * p.mul[s]) hit |= 1u << s;
+  }
+  return hit;
 }
 
 // All level vectors v in [v0, v1) of the current partition (L = 4).
@@ -414,91 +452,170 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                          fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
   int nref = 0;
   const uint32_t s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
-  // Every rare path of the tile loop (unit-boundary tiles, exact corners,
-  // slow re-checks) is entered warp-uniformly (a vote), so the common
-  // iteration carries no convergence-barrier bookkeeping; lanes without work
-  // in a rare path skip it inside.
-  for (uint32_t st = s_lo; st <= s_hi; st++) {
-    const uint32_t j = 2 * st + h;
-    const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
-    const bool live = j < (uint32_t)nloop && vt + 64 > v0 && vt < v1;
-    const bool part = live && (vt < v0 || vt + 64 > v1);
-    if (__any_sync(0xffffffffu, part)) {  // partial tiles at a unit boundary
-      if (part)
+  if constexpr (!ws_has_b0<WS>()) {
+    // sets without b = 0 weights (the c4 bench set): the plain loop; its rare
+    // paths are divergent calls (measured faster here than vote-guarded ones:
+    // c4 slice 639 vs 700 ms)
+    for (uint32_t st = s_lo; st <= s_hi; st++) {
+      const uint32_t j = 2 * st + h;
+      const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
+      if (j >= (uint32_t)nloop || vt + 64 <= v0 || vt >= v1) continue;
+      const float2 lp = wp.lp[j];
+      const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
+      if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
         nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
-      thr_from_sm<WS>(p, thr, thr_sm);
-    }
-    const bool full = live && !part;
-    const float2 lp = wp.lp[j < (uint32_t)nloop ? j : 0u];
-    const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
-    unsigned hitm = 0;
-    float cE, cT;
-    if constexpr (WS::N > 0) {
-      // every configuration's (T, E), min-reduced over the tile: the tile's
-      // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
-      // corner's proxies bound every configuration's from below (a tile
-      // whose corner misses every threshold holds no candidate); a tile that
-      // is not cleared is re-checked configuration by configuration.
-      float mT = __int_as_float(0x7f800000), mE = mT;
-#pragma unroll
-      for (int a = 0; a < 4; a++) {
-        const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
-#pragma unroll
-        for (int b = 0; b < 4; b++) {
-          const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
-#pragma unroll
-          for (int c = 0; c < 4; c++) {
-            const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
-            mT = fminf(mT, T);
-            mE = fminf(mE, E);
+        thr_from_sm<WS>(p, thr, thr_sm);
+        continue;
+      }
+      unsigned hitm = 0;
+      float cE, cT;
+      if constexpr (WS::N > 0) {
+        // every configuration's (T, E), min-reduced over the tile: the tile's
+        // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
+        // corner's proxies bound every configuration's from below (a tile
+        // whose corner misses every threshold holds no candidate); a tile that
+        // is not cleared is re-checked configuration by configuration.
+        float mT = __int_as_float(0x7f800000), mE = mT;
+  #pragma unroll
+        for (int a = 0; a < 4; a++) {
+          const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
+  #pragma unroll
+          for (int b = 0; b < 4; b++) {
+            const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
+  #pragma unroll
+            for (int c = 0; c < 4; c++) {
+              const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
+              mT = fminf(mT, T);
+              mE = fminf(mE, E);
+            }
+          }
+        }
+        if constexpr (WS::RT) {
+          hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
+        } else {
+          float mq[WS::N];
+          WS::q(mT, mE, mq);
+  #pragma unroll
+          for (int s = 0; s < WS::N; s++)
+            if (mq[s] <= thr.vm[s]) hitm |= 1u << s;
+        }
+        cE = mE;
+        cT = mT;
+      } else {  // Pareto only: per-configuration E, min-reduced
+        cT = fmaxf(Tp, minTin);
+        cE = __int_as_float(0x7f800000);
+  #pragma unroll
+        for (int a = 0; a < 4; a++) {
+          const float E1 = Ep + Ae[a];
+  #pragma unroll
+          for (int b = 0; b < 4; b++) {
+            const float E2 = E1 + Be[b];
+  #pragma unroll
+            for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
           }
         }
       }
-      if constexpr (WS::RT) {
-        for (int s = 0; s < p.nw; s++)
-          if (rt_q(p, s, mT, mE) <= thr_sm[s] * p.mul[s]) hitm |= 1u << s;
-      } else {
-        float mq[WS::N];
-        WS::q(mT, mE, mq);
-#pragma unroll
-        for (int s = 0; s < WS::N; s++)
-          if (mq[s] <= thr.vm[s]) hitm |= 1u << s;
+      hitm &= ~b0skip;
+      double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
+      if ((p.b0mode & 2) && hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
+        c64 = tile_corner64(wp, vt);
+        hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
       }
-      cE = mE;
-      cT = mT;
-    } else {  // Pareto only: per-configuration E, min-reduced
-      cT = fmaxf(Tp, minTin);
-      cE = __int_as_float(0x7f800000);
-#pragma unroll
-      for (int a = 0; a < 4; a++) {
-        const float E1 = Ep + Ae[a];
-#pragma unroll
-        for (int b = 0; b < 4; b++) {
-          const float E2 = E1 + Be[b];
-#pragma unroll
-          for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
+      const bool hit = hitm != 0;
+      bool par = false;
+      if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
+        par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
+      if (hit || par) {
+        nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+        thr_from_sm<WS>(p, thr, thr_sm);
+      }
+    }
+  } else {
+    // Every rare path of the tile loop (unit-boundary tiles, exact corners,
+    // slow re-checks) is entered warp-uniformly (a vote), so the common
+    // iteration carries no convergence-barrier bookkeeping; lanes without work
+    // in a rare path skip it inside.
+    for (uint32_t st = s_lo; st <= s_hi; st++) {
+      const uint32_t j = 2 * st + h;
+      const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
+      const bool live = j < (uint32_t)nloop && vt + 64 > v0 && vt < v1;
+      const bool part = live && (vt < v0 || vt + 64 > v1);
+      if (__any_sync(0xffffffffu, part)) {  // partial tiles at a unit boundary
+        if (part)
+          nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
+        thr_from_sm<WS>(p, thr, thr_sm);
+      }
+      const bool full = live && !part;
+      const float2 lp = wp.lp[j < (uint32_t)nloop ? j : 0u];
+      const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
+      unsigned hitm = 0;
+      float cE, cT;
+      if constexpr (WS::N > 0) {
+        // every configuration's (T, E), min-reduced over the tile: the tile's
+        // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
+        // corner's proxies bound every configuration's from below (a tile
+        // whose corner misses every threshold holds no candidate); a tile that
+        // is not cleared is re-checked configuration by configuration.
+        float mT = __int_as_float(0x7f800000), mE = mT;
+  #pragma unroll
+        for (int a = 0; a < 4; a++) {
+          const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
+  #pragma unroll
+          for (int b = 0; b < 4; b++) {
+            const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
+  #pragma unroll
+            for (int c = 0; c < 4; c++) {
+              const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
+              mT = fminf(mT, T);
+              mE = fminf(mE, E);
+            }
+          }
+        }
+        if constexpr (WS::RT) {
+          hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
+        } else {
+          float mq[WS::N];
+          WS::q(mT, mE, mq);
+  #pragma unroll
+          for (int s = 0; s < WS::N; s++)
+            if (mq[s] <= thr.vm[s]) hitm |= 1u << s;
+        }
+        cE = mE;
+        cT = mT;
+      } else {  // Pareto only: per-configuration E, min-reduced
+        cT = fmaxf(Tp, minTin);
+        cE = __int_as_float(0x7f800000);
+  #pragma unroll
+        for (int a = 0; a < 4; a++) {
+          const float E1 = Ep + Ae[a];
+  #pragma unroll
+          for (int b = 0; b < 4; b++) {
+            const float E2 = E1 + Be[b];
+  #pragma unroll
+            for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
+          }
         }
       }
-    }
-    hitm = full ? (hitm & ~b0skip) : 0u;
-    // exact tile corner (fp64 min makespan) where a screen needs it: b = 0
-    // weights (no configuration of the tile beats the lane's best) and the
-    // Pareto screen when the fp32 staircase test cannot decide
-    const bool b0c = (p.b0mode & 2) && hitm && b0_any<WS>(p, hitm);
-    const bool fpar = full && p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE);
-    bool par = false;
-    if (__any_sync(0xffffffffu, b0c || fpar)) {
-      if (b0c || fpar) {
-        const double c64 = tile_corner64(wp, vt);
-        if (b0c) hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
-        if (fpar) par = !stair_dominated(stair, p, c64, cE);
+      hitm = full ? (hitm & ~b0skip) : 0u;
+      // exact tile corner (fp64 min makespan) where a screen needs it: b = 0
+      // weights (no configuration of the tile beats the lane's best) and the
+      // Pareto screen when the fp32 staircase test cannot decide
+      const bool b0c = (p.b0mode & 2) && hitm && b0_any<WS>(p, hitm);
+      const bool fpar = full && p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE);
+      bool par = false;
+      if (__any_sync(0xffffffffu, b0c || fpar)) {
+        if (b0c || fpar) {
+          const double c64 = tile_corner64(wp, vt);
+          if (b0c) hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+          if (fpar) par = !stair_dominated(stair, p, c64, cE);
+        }
       }
-    }
-    const bool hit = hitm != 0;
-    const bool slow = hit || par;
-    if (__any_sync(0xffffffffu, slow)) {
-      if (slow) nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
-      thr_from_sm<WS>(p, thr, thr_sm);
+      const bool hit = hitm != 0;
+      const bool slow = hit || par;
+      if (__any_sync(0xffffffffu, slow)) {
+        if (slow) nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+        thr_from_sm<WS>(p, thr, thr_sm);
+      }
     }
   }
   __syncwarp();
@@ -526,7 +643,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
 #pragma unroll
   for (int s = 0; s < (WS::N > 0 ? WS::N : 1); s++) {
     thr_sm[s] = __int_as_float(0x7f800000);
-    if constexpr (!WS::RT) thr.vm[s] = __int_as_float(0x7f800000);
+    thr.vm[s] = __int_as_float(0x7f800000);
     best_init(lb[s]);
   }
   const int nws = WS::RT ? p.nw : WS::N;  // weights searched
