@@ -244,6 +244,19 @@ int sched_unrank_device(sched_handle *h, const sched_query *q, const uint64_t *d
                         uint64_t advance, int8_t *d_group_of, int8_t *d_level_of, void *ws,
                         size_t ws_bytes, void *stream);
 
+/* Debug / verification entry (tests/test_gpu_scores32.py): runs the PER_GPU
+ * tile kernel (the bench's path; query must be PER_GPU with 4 searched
+ * levels, G <= 8) over the query's window [index_lo, index_hi) (at most 2^26
+ * configurations) with the weight (1,1) and no Pareto set, and writes every
+ * configuration's fp32 hot-loop score as the kernel computes it:
+ * d_scores[2 (i - index_lo)] = T / T_seq and [2 (i - index_lo) + 1] =
+ * E / E_seq (fp32, normalised by the sequential baselines).
+ * Configurations of memory-infeasible partitions are not written (pre-fill).
+ * d_scores is a DEVICE pointer owned by the caller; synchronous.
+ * SCHED_E_INVALID if the query does not run on the tile kernel. */
+int sched_debug_scores32(sched_handle *h, const sched_query *q, void *ws, size_t ws_bytes, void *stream,
+                         float *d_scores);
+
 /* fp64 canonical score of one configuration on the host, weight w (0..W-1;
  * with W == 0 score64 = X).  out->valid = 0 if memory-infeasible.  Host only. */
 int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int32_t w,

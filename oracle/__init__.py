@@ -213,6 +213,20 @@ def search_parallel(prof, q, procs: int | None = None, windows: int | None = Non
     return merge(parts, q.want_pareto)
 
 
+def score_window(prof, q):
+    """fp64 canonical (T, E) of every configuration of [q.index_lo,
+    q.index_hi) in index order (NaN where infeasible): two numpy arrays."""
+    pk = _Pack(prof, q)
+    n = int(pk.Q.hi - pk.Q.lo)
+    T = np.empty(n, np.float64)
+    E = np.empty(n, np.float64)
+    f = lib().oracle_score_window
+    f.restype = C.c_uint64
+    got = f(C.byref(pk.P), C.byref(pk.Q), _ptr(T, C.c_double), _ptr(E, C.c_double))
+    assert got == n
+    return T, E
+
+
 def config(q, idx: int):
     """Index -> (RGS a[n], level digits) by the oracle's own enumeration."""
     a = (C.c_int * 64)()

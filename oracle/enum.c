@@ -295,6 +295,8 @@ typedef struct {
   uint64_t ncfg, nfeas;
   /* single-config extraction */
   int extract; uint64_t want; int *out_a, *out_lv; int got;
+  /* window scores: (T, E) of every configuration of [lo, hi), NaN if infeasible */
+  double *outT, *outE;
 } ctx_t;
 
 static void pareto_add(ctx_t *C, uint64_t idx, double T, double E) {
@@ -332,8 +334,12 @@ static void leaf(ctx_t *C, int k, uint64_t base) {
     }
     C->ncfg++;
     double T, E;
-    if (!oracle_score_config(C->P, q, q->n, C->a, k, pl, &T, &E)) continue;
+    if (!oracle_score_config(C->P, q, q->n, C->a, k, pl, &T, &E)) {
+      if (C->outT) { C->outT[idx - q->lo] = __builtin_nan(""); C->outE[idx - q->lo] = __builtin_nan(""); }
+      continue;
+    }
     C->nfeas++;
+    if (C->outT) { C->outT[idx - q->lo] = T; C->outE[idx - q->lo] = E; }
     for (int w = 0; w < q->nw; w++) {
       double F = objective(C->tseq, C->eseq, T, E, q->wa[w], q->wb[w]);
       if (!C->best[w].found || F > C->best[w].f) {   /* strict: lowest index wins ties */
@@ -380,6 +386,24 @@ int oracle_search(const or_profile *P, const or_query *q, int l100,
   int ovf = C->par_overflow;
   free(C);
   return ovf ? -4 : 0;
+}
+
+/* fp64 canonical (T, E) of every configuration of the window [q->lo, q->hi)
+ * into outT / outE (index - lo; NaN if infeasible), same enumeration as
+ * oracle_search.  Returns the number of configurations. */
+uint64_t oracle_score_window(const or_profile *P, const or_query *q, double *outT, double *outE) {
+  ctx_t *C = calloc(1, sizeof(ctx_t));
+  C->P = P; C->q = q; C->outT = outT; C->outE = outE;
+  or_best dummy[8];
+  C->best = dummy;
+  or_query q2 = *q; q2.nw = 0; q2.want_pareto = 0;
+  C->q = &q2;
+  count_setup(&q2);
+  C->a[0] = 0; C->sz[0] = 1;
+  if (q2.n >= 1 && q2.lo < q2.hi) rec(C, 1, 1, 0);
+  uint64_t n = C->ncfg;
+  free(C);
+  return n;
 }
 
 /* Decode index -> (RGS a[n], level digits lv[n or k]); returns k or -1. */

@@ -402,6 +402,45 @@ int sched_unrank_device(sched_handle *h, const sched_query *qin, const uint64_t 
   GUARD_END
 }
 
+int sched_debug_scores32(sched_handle *h, const sched_query *qin, void *ws, size_t ws_bytes, void *stream,
+                         float *d_scores) {
+  GUARD_BEGIN
+  if (!h || !qin || !ws || !d_scores) return SCHED_E_INVALID;
+  int st = need_device();
+  if (st) return st;
+  sched_query qq = *qin;
+  const int32_t w11[2] = {1, 1};
+  qq.weights = w11;
+  qq.n_weights = 1;
+  qq.want_pareto = 0;
+  Query q;
+  const Space *sp;
+  st = resolve(h, &qq, &q, &sp);
+  if (st) return st;
+  if (q.hi - q.lo > ((uint64_t)1 << 26)) return SCHED_E_INVALID;
+  std::vector<unsigned char> blob;
+  DevParams dp;
+  st = build_stage(h->P, q, *sp, &blob, &dp);
+  if (st) return st;
+  if (ws_bytes < workspace_bytes(dp, 0) || ((uintptr_t)ws & 255)) return SCHED_E_WORKSPACE;
+  if (h->staged_ws != ws || h->staged_blob != blob) {
+    st = do_stage(h, dp, blob, ws, stream);
+    if (st) return st;
+  }
+  dp.dump = (unsigned char *)d_scores;
+  dp.dump_lo = q.lo;
+  dp.dump_n = q.hi - q.lo;
+  LaunchInfo info;
+  std::vector<BestRec> bres;
+  std::vector<CandRec> front;
+  uint64_t ctr[kCtrN];
+  st = launch_search(dp, ws, ws_bytes, stream, &info, &bres, &front, ctr);
+  if (st) return st;
+  if (info.path != 1) return SCHED_E_INVALID;
+  return SCHED_OK;
+  GUARD_END
+}
+
 int sched_score(const sched_handle *hc, const sched_query *qin, uint64_t index, int32_t w, sched_pick *out) {
   GUARD_BEGIN
   if (!hc || !out) return SCHED_E_INVALID;

@@ -115,6 +115,8 @@ struct DevParams {
   int gtab_ok;                 // workspace holds a group table for this query
   int b0mode;                  // tile kernel, weights with b = 0: bit 0 partition-level, bit 1 tile-level
                                // early reject (default 3; SCHED_B0 overrides, measurement only)
+  unsigned char *dump;         // sched_debug_scores32: float2 (T-hat, E-hat) per configuration of
+  uint64_t dump_lo, dump_n;    // [dump_lo, dump_lo + dump_n) (nullptr: no dump)
   const DevParams *gp;         // this block's copy in the workspace (global memory): handed to the
                                // out-of-line slow paths, so no thread copies the kernel parameters
                                // to its stack (local memory)

@@ -24,6 +24,7 @@ namespace sched {
 // ---- compile-time product-metric sets: q_s = (T/T_seq)^a (E/E_seq)^b ----
 struct WS_P {  // Pareto only
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 0;
   __host__ __device__ static constexpr int A(int s) { return 0; }
   __host__ __device__ static constexpr int B(int s) { return 0; }
@@ -31,6 +32,7 @@ struct WS_P {  // Pareto only
 };
 struct WS_11 {
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 1; }
   __host__ __device__ static constexpr int B(int s) { return 1; }
@@ -38,6 +40,7 @@ struct WS_11 {
 };
 struct WS_10 {
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 1; }
   __host__ __device__ static constexpr int B(int s) { return 0; }
@@ -45,6 +48,7 @@ struct WS_10 {
 };
 struct WS_01 {
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 1;
   __host__ __device__ static constexpr int A(int s) { return 0; }
   __host__ __device__ static constexpr int B(int s) { return 1; }
@@ -52,6 +56,7 @@ struct WS_01 {
 };
 struct WS_11_21 {  // c4: [T x E], [T x T x E]
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 2;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : 2); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 1 : 1); }
@@ -62,6 +67,7 @@ struct WS_11_21 {  // c4: [T x E], [T x T x E]
 };
 struct WS_C1 {  // (1,0) (0,1) (1,1) (2,1)
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 4;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : (s == 1 ? 0 : (s == 2 ? 1 : 2))); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 0 : (s == 1 ? 1 : (s == 2 ? 1 : 1))); }
@@ -74,6 +80,7 @@ struct WS_C1 {  // (1,0) (0,1) (1,1) (2,1)
 };
 struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
   static constexpr bool RT = false;
+  static constexpr bool DUMP = false;
   static constexpr int N = 7;
   __host__ __device__ static constexpr int A(int s) { return (s == 0 ? 1 : (s == 1 ? 3 : (s == 2 ? 2 : (s == 3 ? 1 : (s == 4 ? 1 : (s == 5 ? 1 : 0)))))); }
   __host__ __device__ static constexpr int B(int s) { return (s == 0 ? 0 : (s == 1 ? 1 : (s == 2 ? 1 : (s == 3 ? 1 : (s == 4 ? 2 : (s == 5 ? 3 : 1)))))); }
@@ -97,10 +104,25 @@ struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
 struct WS_RT {
   static constexpr int N = kMaxW;
   static constexpr bool RT = true;
+  static constexpr bool DUMP = false;
   __host__ __device__ static constexpr int A(int) { return 0; }
   __host__ __device__ static constexpr int B(int) { return 0; }
   __device__ static __forceinline__ void q(float, float, float *) {}
 };
+
+// WS_11 that also writes every configuration's fp32 (T-hat, E-hat), as the
+// tile loop computes them, to p.dump (sched_debug_scores32: the hot loop's
+// fp32 scores checked against the oracle configuration by configuration)
+struct WS_11_DUMP : WS_11 {
+  static constexpr bool DUMP = true;
+};
+
+template <class WS>
+__device__ __forceinline__ void dump_score(const DevParams &p, u64 idx, float T, float E) {
+  if constexpr (WS::DUMP) {
+    if (idx >= p.dump_lo && idx - p.dump_lo < p.dump_n) ((float2 *)p.dump)[idx - p.dump_lo] = make_float2(T, E);
+  }
+}
 
 // q_s = (T/T_seq)^a (E/E_seq)^b for query weight s, run-time exponents
 __device__ __forceinline__ float rt_q(const DevParams &p, int s, float T, float E) {
@@ -290,6 +312,7 @@ __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, c
       E += wp.ge[b * 4 + dig[b]];
       T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
+    dump_score<WS>(p, wp.base + v, T, E);
     if constexpr (WS::RT) {
       for (int s = 0; s < p.nw; s++) thr[s] = fminf(thr[s], rt_q(p, s, T, E));
     } else if constexpr (WS::N > 0) {
@@ -487,6 +510,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
               const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
+              dump_score<WS>(p, wp.base + vt + (uint32_t)(a * 16 + b * 4 + c), T, E);
             }
           }
         }

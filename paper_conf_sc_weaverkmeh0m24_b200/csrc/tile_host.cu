@@ -26,6 +26,11 @@ static bool ws_match(const DevParams &dp, int *perm) {
 template <int L>
 static const void *tile_pick_ws(DevParams *dp) {
   int perm[kMaxW];
+  if (dp->dump) {  // sched_debug_scores32: the (1,1) kernel that also dumps every configuration's fp32 score
+    if (dp->nw != 1 || dp->wa[0] != 1 || dp->wb[0] != 1) return nullptr;
+    dp->ws_perm[0] = 0;
+    return tile_fn<L, WS_11_DUMP>();
+  }
   // SCHED_TILE_RT=1 (measurement): the run-time-weight variant even where a
   // compiled-in weight set matches
   const char *rt = std::getenv("SCHED_TILE_RT");

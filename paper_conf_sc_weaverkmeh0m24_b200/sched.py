@@ -34,7 +34,8 @@ UINT64_MAX = (1 << 64) - 1
 EXPORTS = ["sched_create", "sched_destroy", "sched_count", "sched_workspace_size", "sched_stage",
            "sched_search", "sched_merge", "sched_unrank", "sched_rank", "sched_score", "sched_heuristic",
            "sched_strerror", "sched_version", "sched_dp_workspace_size", "sched_front_dp",
-           "sched_split_workspace_size", "sched_search_splits", "sched_unrank_device"]
+           "sched_split_workspace_size", "sched_search_splits", "sched_unrank_device",
+           "sched_debug_scores32"]
 
 
 class SchedError(RuntimeError):
@@ -320,6 +321,21 @@ class Scheduler:
                                          C.c_void_p(lv.data_ptr()), C.c_void_p(ws.data_ptr()),
                                          C.c_size_t(ws.numel()), C.c_void_p(st)), "sched_unrank_device")
         return g, lv
+
+    def debug_scores32(self, q, stream=None):
+        """fp32 hot-loop (T/T_seq, E/E_seq) of every configuration of q's
+        window on the tile kernel (sched_debug_scores32); NaN rows where the
+        partition is memory-infeasible.  Returns a float32 device tensor [n, 2]."""
+        import torch
+        n = int(q.index_hi) - int(q.index_lo)
+        out = torch.full((n, 2), float("nan"), dtype=torch.float32, device="cuda")
+        qq = dataclasses.replace(q, weights=((1, 1),), want_pareto=False)
+        ws = self.workspace(qq)
+        st = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        _check(lib().sched_debug_scores32(self._h, C.byref(self.cquery(qq)), C.c_void_p(ws.data_ptr()),
+                                          C.c_size_t(ws.numel()), C.c_void_p(st), C.c_void_p(out.data_ptr())),
+               "sched_debug_scores32")
+        return out
 
     def score(self, q, index, w=0) -> Pick:
         out = Pick()

@@ -178,3 +178,23 @@ def test_min_makespan_subset_dp():
         minT = min(dp[full].values())
         assert r["best"][0][2] == pytest.approx(minT, rel=1e-12)
         assert r["best"][0][1] == pytest.approx(r["tseq"] / minT, rel=1e-12)
+
+
+def test_score_window_equals_per_index_scoring():
+    """oracle.score_window (every configuration of a window, enumeration
+    order) == oracle.config + oracle.score index by index (the extraction
+    path), NaN exactly where infeasible."""
+    import math
+    import oracle
+    from synth import make_profile, Query, PER_GPU, PER_CLIENT
+    for scope, arch in ((PER_GPU, [11, 2, 0, 12, 5, 1, 3]), (PER_CLIENT, None)):
+        prof = make_profile(7 if arch else 6, levels=(25, 50, 75, 100), seed=41, archetypes=arch)
+        q = Query(prof.n_workflows, 3, 4, (50, 100), scope, ((1, 1),), False)
+        lo, hi = 37, 37 + 700
+        T, E = oracle.score_window(prof, q.with_range(lo, hi))
+        for i in range(lo, hi):
+            ok, t, e = oracle.score(prof, q, *oracle.config(q, i))
+            if ok:
+                assert (T[i - lo], E[i - lo]) == (t, e)
+            else:
+                assert math.isnan(T[i - lo]) and math.isnan(E[i - lo])
