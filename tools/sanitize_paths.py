@@ -24,6 +24,8 @@ CASES = [  # name, SCHED_KERNEL, expected path, n, g, c, levels, scope, weights,
     ("ctile", "ctile", 5, 7, 3, 7, (25, 50, 75, 100), PER_CLIENT, W, 3),
     ("sfx", "sfx", 3, 10, 5, 3, (100,), PER_GPU, SWEEP, 4),
     ("dfs", "dfs", 2, 10, 5, 3, (100,), PER_GPU, SWEEP, 4),
+    ("ctile2", "ctile2", 6, 7, 4, 3, (25, 50, 75, 100), PER_CLIENT, W, 7),        # round 2: group-table PER_CLIENT
+    ("tile_rt", "tile", 1, 9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 2), (3, 1), (1, 0)), 8),   # run-time weights
 ]
 
 
@@ -54,6 +56,32 @@ if not ONLY or "front_dp" in ONLY:
     ref = oracle.search(prof, q)
     assert sorted((p.makespan_s, p.energy_j) for p in front) == sorted((t, e) for _, t, e in ref["pareto"])
     print(f"front_dp: ok ({len(front)} points)", flush=True)
+
+if not ONLY or "unrank_device" in ONLY:
+    import torch
+    prof = make_profile(8, levels=(25, 50, 75, 100), seed=9)
+    q = Query(8, 4, 8, (25, 50, 75, 100), PER_GPU, W, True)
+    sch = S.Scheduler(prof)
+    idx = torch.arange(0, S.count(q), 97, dtype=torch.int64)
+    g, lv = sch.unrank_device(q, idx, advance=3)
+    g = g.cpu().tolist()
+    for t in range(0, len(g), 50):
+        i = int(idx[t]) + 3
+        if i < S.count(q):
+            assert g[t] == oracle.config(q, i)[0]
+    print("unrank_device: ok", flush=True)
+
+if not ONLY or "scores32" in ONLY:
+    import math
+    prof = make_profile(9, levels=(25, 50, 75, 100), seed=10)
+    q = Query(9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 1),), False, 1000, 21000)
+    out = S.Scheduler(prof).debug_scores32(q).cpu().tolist()
+    T, E = oracle.score_window(prof, q)
+    ts, es = oracle.constants(prof, q)
+    for k in range(0, 20000, 37):
+        if not math.isnan(T[k]):
+            assert abs(out[k][0] / (T[k] / ts) - 1) <= 1e-5
+    print("debug_scores32: ok", flush=True)
 
 if not ONLY or "splits" in ONLY:
     prof = make_profile(3, levels=(50, 100), seed=6)
