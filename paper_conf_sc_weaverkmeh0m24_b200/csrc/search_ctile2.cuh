@@ -298,6 +298,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
       const bool feas = wp.cfg.feasible;
       const uint32_t v0 = s > base ? (uint32_t)(s - base) : 0u;
       const uint32_t v1 = e - base < (u64)Pn ? (uint32_t)(e - base) : Pn;
+      __syncwarp();  // every lane has read the partition descriptor before lane 0 updates the warp's counters
       if (lane == 0) {
         wp.ncfg += v1 - v0;
         if (feas) wp.nfeas += v1 - v0;
