@@ -29,6 +29,18 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
   if (err != cudaSuccess) return err;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   *grid = std::min(4096, nsm * occ);
+  if (fixed_units && dp.chunk_log2 >= 12) {
+    // seed pass: a unit smaller than a partition fixes only the top index
+    // digits, so a tile whose client is a low-numbered workflow straddles it
+    // and goes configuration by configuration; sample 4 units of up to 2^20
+    // configurations per SM instead of 128 of 2^10 (c3-client slice: the
+    // seed pass 60 -> ~2 ms)
+    const int sl = std::min(20, dp.chunk_log2);
+    const uint64_t units = dp.n_owned << (dp.chunk_log2 - sl);
+    dp.unit_log2 = sl;
+    dp.n_units = std::min<uint64_t>(units, (uint64_t)nsm * 4);
+    dp.unit_stride = std::max<uint64_t>(1, units / std::max<uint64_t>(1, dp.n_units));
+  }
   if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kC2Warps;

@@ -43,5 +43,6 @@ for s in a.sets.split(","):
         print(json.dumps({"workload": a.name, "set": s, "rep": r, "path": st["kernel_path"],
                           "search_ms": st["search_ms"], "configs": st["n_configs"],
                           "configs_per_s": st["n_configs"] / (st["search_ms"] / 1e3),
-                          "refined": st["n_refined"], "cand": st["n_candidates"], "status": res.status}),
+                          "refined": st["n_refined"], "cand": st["n_candidates"], "status": res.status,
+                          "passes": st["passes"], "launches": st["kernel_launches"], "total_ms": st["total_ms"]}),
               flush=True)
