@@ -10,6 +10,8 @@ static size_t ctile2_smem(const DevParams &dp) {
   return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(C2Warp) * kC2Warps + sizeof(BestRec) * kC2Warps * kMaxW;
 }
 
+size_t ctile2_t64_bytes() { return sizeof(double) * (size_t)kC2MaxGrid * kC2Warps * kC2Tab; }
+
 bool ctile2_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.scope != SCHED_PER_CLIENT || dp.L != 4 || dp.n < 6 || dp.n > 15 || dp.g > 8) return false;
   if (dp.c > 4) return false;  // groups of <= 4 clients: tables <= 836 entries
@@ -28,19 +30,7 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
   err = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tl.fn, kC2Threads, tl.smem);
   if (err != cudaSuccess) return err;
   if (occ < 1) return cudaErrorInvalidConfiguration;
-  *grid = std::min(4096, nsm * occ);
-  if (fixed_units && dp.chunk_log2 >= 12) {
-    // seed pass: a unit smaller than a partition fixes only the top index
-    // digits, so a tile whose client is a low-numbered workflow straddles it
-    // and goes configuration by configuration; sample 4 units of up to 2^20
-    // configurations per SM instead of 128 of 2^10 (c3-client slice: the
-    // seed pass 60 -> ~2 ms)
-    const int sl = std::min(20, dp.chunk_log2);
-    const uint64_t units = dp.n_owned << (dp.chunk_log2 - sl);
-    dp.unit_log2 = sl;
-    dp.n_units = std::min<uint64_t>(units, (uint64_t)nsm * 4);
-    dp.unit_stride = std::max<uint64_t>(1, units / std::max<uint64_t>(1, dp.n_units));
-  }
+  *grid = std::min(kC2MaxGrid, nsm * occ);
   if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kC2Warps;

@@ -117,6 +117,7 @@ struct DevParams {
                                // early reject (default 3; SCHED_B0 overrides, measurement only)
   unsigned char *dump;         // sched_debug_scores32: float2 (T-hat, E-hat) per configuration of
   uint64_t dump_lo, dump_n;    // [dump_lo, dump_lo + dump_n) (nullptr: no dump)
+  double *c2t64;               // k_ctile2: per-warp exact fp64 T_g table (global, [grid][warps][tab])
   const DevParams *gp;         // this block's copy in the workspace (global memory): handed to the
                                // out-of-line slow paths, so no thread copies the kernel parameters
                                // to its stack (local memory)

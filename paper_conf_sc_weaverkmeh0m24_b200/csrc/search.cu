@@ -495,7 +495,7 @@ constexpr int kMaxGrid = 4096;
 constexpr int kFrontCap = 1 << 16;
 
 struct WsLayout {
-  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, fin, out, gtab, params, total;
+  size_t ctr, thr, stv, stp, ste, stlog, blob, slots, cand, surv, fin, out, gtab, params, c2t64, total;
 };
 
 WsLayout layout(const DevParams &dp) {
@@ -519,6 +519,11 @@ WsLayout layout(const DevParams &dp) {
   L.surv = take(4 * (size_t)dp.cand_cap);
   L.fin = take(finalize_bytes(dp.cand_cap));
   L.params = take(sizeof(DevParams));
+  {  // per-warp fp64 T tables of the group-table PER_CLIENT kernel (only when it runs)
+    DevParams tmp = dp;
+    TileLaunch tl;
+    L.c2t64 = take(ctile2_eligible(tmp, &tl) && dp.want_pareto ? ctile2_t64_bytes() : 0);
+  }
   L.out = take(sizeof(BestRec) * kMaxW + sizeof(CandRec) * (size_t)kFrontCap);
   L.gtab = take(dp.gtab_ok ? sizeof(GroupRec) * ((size_t)dp.L << dp.n) : 0);
   L.total = (o + 255) / 256 * 256;
@@ -614,6 +619,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
   dp.out = ws + L.out;
   dp.gtab = dp.gtab_ok ? ws + L.gtab : nullptr;
   dp.gp = (const DevParams *)(ws + L.params);
+  dp.c2t64 = (double *)(ws + L.c2t64);
   int dev = 0, nsm = 0;
   CK(cudaGetDevice(&dev));
   CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev));

@@ -38,7 +38,8 @@ constexpr int kC2Threads = 512;
 constexpr int kC2Warps = kC2Threads / 32;
 constexpr int kC2Tab = 896;    // table entries per warp: 4 pad + sum_g roundup4(4^|g|) <= 4 + 3*256 + 64
 constexpr int kC2Bits = 20;    // bits of st: 4^(n-3) / 32 <= 2^19 for n <= 15
-constexpr int kC2Slots = 8;    // 5 fixed-group slots + A, B, C; slot 8 of the delta rows = vo
+constexpr int kC2Slots = 8;
+constexpr int kC2MaxGrid = 256;  // CTAs (1 per SM): bounds the workspace's fp64 T tables    // 5 fixed-group slots + A, B, C; slot 8 of the delta rows = vo
 
 struct C2Warp {
   LaneCfg cfg;
@@ -64,23 +65,37 @@ __device__ __forceinline__ void c2_offsets(const C2Warp &wp, int *off) {
   for (int g = 0; g < wp.cfg.k; g++) off[g + 1] = off[g] + (((1 << (2 * __popc(wp.cfg.mask[g]))) + 3) & ~3);
 }
 
-// per-partition group tables (fp32 T-hat, E-hat at every member-level vector)
-__device__ __forceinline__ void c2_tables(const Tables &tb, const DevParams &p, C2Warp &wp, int lane) {
+// per-partition group tables: fp32 (T-hat, E-hat) at every member-level
+// vector in shared memory, and the exact canonical fp64 T_g (refine64 order)
+// in the warp's global table t64 (read only by the tile's exact-corner
+// Pareto check, through L2)
+__device__ __forceinline__ void c2_tables(const Tables &tb, const DevParams &p, C2Warp &wp, int lane,
+                                          double *t64) {
   const int k = wp.cfg.k;
   int off[kMaxG + 1];
   c2_offsets(wp, off);
   for (int e = lane; e < off[k]; e += 32) {
     float2 v = make_float2(0.f, 0.f);
+    double T64 = 0.0;
     if (e >= 4) {
       int g = 0;
       while (e >= off[g + 1]) g++;
       const uint32_t m = wp.cfg.mask[g];
       const int s = __popc(m);
       const uint32_t var = (uint32_t)(e - off[g]);
-      if (var < (1u << (2 * s))) ct_group32(tb, p, m, c2_lw(m, var, s), v.x, v.y);
+      if (var < (1u << (2 * s))) {
+        const uint32_t lw = c2_lw(m, var, s);
+        ct_group32(tb, p, m, lw, v.x, v.y);
+        if (p.want_pareto) {
+          double E64;
+          ct_group64(tb, p, m, lw, T64, E64);
+        }
+      }
     }
     wp.tab[e] = v;
+    if (p.want_pareto) __stcg(t64 + e, T64);
   }
+  __threadfence_block();
   __syncwarp();
 }
 
@@ -264,6 +279,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
   int nref = 0;
   const int n = p.n;
   const int ul = p.unit_log2, cl = p.chunk_log2;
+  double *t64 = p.c2t64 + ((size_t)blockIdx.x * kC2Warps + warp) * kC2Tab;
 
   for (;;) {
     u64 unit = 0;
@@ -306,7 +322,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
       if (feas) {
         int idxL[kC2Slots];
         uint32_t voL, tbits;
-        c2_tables(tb, p, wp, lane);
+        c2_tables(tb, p, wp, lane, t64);
         if (k < 3) {
           nref += c2_small<WM>(tb, *p.gp, stair, wp, thr, lb, v0, v1, lane);
         } else {
@@ -401,7 +417,18 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
                   hit |= q <= thr[w] * p.mul[w];
                 }
               }
-              const bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+              bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+              if (par) {  // the fp32 screen cannot decide: the tile's exact fp64 corner makespan
+                double c = 0.0;
+#pragma unroll
+                for (int q = 0; q < 5; q++) c = fmax(c, __ldcg(t64 + idxS[q] + idxL[q]));
+#pragma unroll
+                for (int q = 5; q < 8; q++) {
+                  const double *tq = t64 + idxS[q] + idxL[q];
+                  c = fmax(c, fmin(fmin(__ldcg(tq), __ldcg(tq + 1)), fmin(__ldcg(tq + 2), __ldcg(tq + 3))));
+                }
+                par = !stair_dominated(stair, p, c, mE);
+              }
               if (!hit && !par) continue;
             }
             nref += c2_tile_slow<WM>(tb, *p.gp, stair, wp, thr, lb, o, vo, v0, v1, Tp, Ep, At, Ae, Bt, Be, Ct, Ce);

@@ -49,6 +49,7 @@ bool dfs_eligible(DevParams &dp, TileLaunch *tl);
 bool sfx_eligible(DevParams &dp, TileLaunch *tl);
 bool ctile_eligible(DevParams &dp, TileLaunch *tl);
 bool ctile2_eligible(DevParams &dp, TileLaunch *tl);
+size_t ctile2_t64_bytes();
 cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,
                           cudaEvent_t e2, int *grid, bool fixed_units);
 cudaError_t launch_ctile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream_t st, cudaEvent_t e1,

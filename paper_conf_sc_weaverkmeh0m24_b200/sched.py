@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_HERE, "libsched.so")
+SO_PATH = os.environ.get("SCHED_SO_PATH") or os.path.join(_HERE, "libsched.so")  # override: A/B measurements
 
 SCHED_OK = 0
 SCHED_E_INVALID = -1
