@@ -2,6 +2,9 @@
 // kernel (search_ctile2.cuh, kernel_path 6): PER_CLIENT scope, L = 4,
 // 6 <= n <= 15, groups of <= 4 clients (C <= 4), G <= 8, canonical model or
 // POWER_CAP (E = sum_g E_g, level-independent feasibility).
+#include <cstdio>
+#include <cstdlib>
+
 #include "search_ctile2.cuh"
 
 namespace sched {
@@ -31,6 +34,19 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
   if (err != cudaSuccess) return err;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   *grid = std::min(kC2MaxGrid, nsm * occ);
+  if (fixed_units && dp.chunk_log2 >= 12) {
+    // seed pass: units smaller than a partition fix only the top index
+    // digits, and a tile whose client is a low-numbered workflow straddles
+    // such a unit (configuration-by-configuration path); sample
+    // per_sm x nsm units of 2^ul configurations (SCHED_C2_SEED="ul,per_sm")
+    int sl = 16, per = 32;
+    if (const char *e = std::getenv("SCHED_C2_SEED")) std::sscanf(e, "%d,%d", &sl, &per);
+    sl = std::max(10, std::min(sl, dp.chunk_log2));
+    const uint64_t units = dp.n_owned << (dp.chunk_log2 - sl);
+    dp.unit_log2 = sl;
+    dp.n_units = std::min<uint64_t>(units, (uint64_t)nsm * std::max(1, per));
+    dp.unit_stride = std::max<uint64_t>(1, units / std::max<uint64_t>(1, dp.n_units));
+  }
   if (!fixed_units) {  // units of 2^12 .. 2^chunk_log2 configs, >= ~8 per warp
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kC2Warps;
