@@ -57,7 +57,6 @@ struct SfxLane {   // per-lane suffix state (registers)
   uint32_t rm;     // bit j: group j has room
   int kc;          // open groups
   float T, E;      // fp32 normalised makespan / energy so far
-  int ds;          // DP count-table state after these placements (fast pass: subtree sizes)
 };
 
 struct SfxHot {    // fast-pass accumulators (registers)
@@ -74,9 +73,6 @@ struct SfxCold {   // slow-pass state (local memory)
 
 struct SfxCtx {    // read-only per-prefix context
   const float2 *tab;
-  const u64 *W;             // DP count table (shared): W[state] = completions below state
-  const uint16_t *trans;    // DP transitions (shared), row stride tc
-  int tc, capped;
   int G, C, start[8];
   int kp, off;     // prefix groups, suffix bit offset (n - M)
   u64 base;
@@ -99,13 +95,6 @@ __device__ __forceinline__ void sfx_apply(SfxLane &s, int j, uint32_t bi, float2
   const uint32_t has = ((s.rr >> (4 * j)) & 15u) ? 1u : 0u;
   s.rm = (s.rm & ~(1u << j)) | (has << j);
   s.gi |= (u64)bi << (8 * j);
-}
-
-// DP state after placing the next element into option j (new group: column
-// 0; an existing group: its size before the join when capped, else column 1)
-__device__ __forceinline__ int sfx_ds(const SfxCtx &x, const SfxLane &s, int j) {
-  const int col = j == s.kc ? 0 : (x.capped ? x.C - (int)((s.rr >> (4 * j)) & 15u) : 1);
-  return x.trans[s.ds * x.tc + col];
 }
 
 // One configuration of the slow pass: fp32 screens, fp64 canonical re-score
@@ -280,39 +269,23 @@ __device__ __forceinline__ void sfx_slots(const float2 *tab, const SfxLane &s, i
 
 // next option at level I (I <= M-2) and the first parent below it; false
 // when level I is exhausted.  st[I] = state before x_I, rem[I] = options left.
-// A memory-infeasible partial configuration (T = +inf) has only infeasible
-// completions: the whole subtree is skipped at once, its size W[ds] taken
-// off the lane's remaining count (it scores nothing feasible and moves no
-// minimum).  cnt = 0 on return: the lane's range ended inside a skipped
-// subtree.
 template <int M, int I>
 __device__ __forceinline__ bool sfx_adv(const SfxCtx &x, SfxLane (&st)[M - 1], uint32_t (&rem)[M - 1],
-                                        SfxLane &par, int &cnt) {
+                                        SfxLane &par) {
   constexpr int RS = SfxWarp<M>::RS;
   while (rem[I]) {
     const int j = __ffs(rem[I]) - 1;
     rem[I] &= rem[I] - 1;
     const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
     SfxLane s = st[I];
-    s.ds = sfx_ds(x, st[I], j);
     sfx_apply(s, j, 1u << I, v, x.C);
-    if (!(s.T < __int_as_float(0x7f800000))) {
-      const u64 wsub = x.W[s.ds];
-      if (wsub >= (u64)cnt) {
-        cnt = 0;
-        return false;
-      }
-      cnt -= (int)wsub;
-      continue;
-    }
     if constexpr (I == M - 2) {
       par = s;
       return true;
     } else {
       st[I + 1] = s;
       rem[I + 1] = sfx_opts(s, x.G);
-      if (sfx_adv<M, I + 1>(x, st, rem, par, cnt)) return true;
-      if (cnt == 0) return false;
+      if (sfx_adv<M, I + 1>(x, st, rem, par)) return true;
     }
   }
   return false;
@@ -320,13 +293,12 @@ __device__ __forceinline__ bool sfx_adv(const SfxCtx &x, SfxLane (&st)[M - 1], u
 
 template <int M, int I>
 __device__ __forceinline__ bool sfx_next(const SfxCtx &x, SfxLane (&st)[M - 1], uint32_t (&rem)[M - 1],
-                                         SfxLane &par, int &cnt) {
-  if (sfx_adv<M, I>(x, st, rem, par, cnt)) return true;
-  if (cnt == 0) return false;
+                                         SfxLane &par) {
+  if (sfx_adv<M, I>(x, st, rem, par)) return true;
   if constexpr (I == 0) {
     return false;
   } else {
-    return sfx_next<M, I - 1>(x, st, rem, par, cnt);
+    return sfx_next<M, I - 1>(x, st, rem, par);
   }
 }
 
@@ -345,7 +317,6 @@ __device__ __forceinline__ void sfx_fast(const DevParams &p, const Stair &stair,
     rem[I] = sfx_opts(st[I], x.G) & (~1u << j);  // options after the start choice
     const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
     SfxLane s = st[I];
-    s.ds = sfx_ds(x, st[I], j);
     sfx_apply(s, j, 1u << I, v, x.C);
     if (I < M - 2) st[I + 1] = s;
     else par = s;
@@ -360,7 +331,7 @@ __device__ __forceinline__ void sfx_fast(const DevParams &p, const Stair &stair,
     if (o == sfx_opts(par, x.G)) sfx_slots<M>(x.tab, par, x.G, h.mT, h.mE, h.nf);
     else sfx_last<M, false>(p, stair, x, h, nullptr, par, o);  // the partial first parent
     cnt -= n;
-    if (!sfx_next<M, M - 2>(x, st, rem, par, cnt)) return;
+    if (!sfx_next<M, M - 2>(x, st, rem, par)) return;
     o = sfx_opts(par, x.G);
   }
 }
@@ -595,10 +566,6 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
         if (l1 > l0) {
           SfxCtx x;
           x.tab = w.tab;
-          x.W = tb.W;
-          x.trans = tb.trans;
-          x.tc = p.tc;
-          x.capped = p.capped;
           x.G = p.g;
           x.C = p.c;
           x.kp = kp;
@@ -612,7 +579,6 @@ __global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
           s0.kc = kp;
           s0.T = Tp;
           s0.E = Ep;
-          s0.ds = w.cfg.st[plen - 1];
           for (int r = 0; r < kp; r++) {
             const int room = min(p.c - (int)w.cfg.sz[r], 15);
             s0.rr |= (uint32_t)room << (4 * r);
