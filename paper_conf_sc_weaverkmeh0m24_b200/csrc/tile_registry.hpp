@@ -29,10 +29,10 @@ struct TileLaunch {
 };
 
 #ifndef SCHED_TILE_THREADS
-#define SCHED_TILE_THREADS 256
+#define SCHED_TILE_THREADS 512
 #endif
 #ifndef SCHED_TILE_MINB
-#define SCHED_TILE_MINB 2
+#define SCHED_TILE_MINB 1
 #endif
 constexpr int kTileThreads = SCHED_TILE_THREADS;
 constexpr int kTileMinBlocks = SCHED_TILE_MINB;  // __launch_bounds__ min blocks per SM
