@@ -414,14 +414,64 @@ __device__ __forceinline__ unsigned rt_screen(const DevParams &p, const Thr<WS> 
   return hit;
 }
 
+// L = 2 or 3 searched levels (any partition) -- the L = 4 tile shape (64
+// configurations of the last three groups in registers, lanes over two more
+// digits) does not apply: every lane takes configurations v0 + lane + 32 i,
+// decodes their base-L level digits and scores them from the partition's
+// group records (T = max, E = sum in block order), screens them (run-time
+// weights: the log-domain pre-screen; Pareto: the fp32 staircase, then the
+// exact fp64 makespan), and sends the rare survivors to check_config.
+template <int L, class WS>
+__device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams &p, const Stair &stair,
+                                               const WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
+                                               uint32_t v0, uint32_t v1, int lane) {
+  const int k = wp.cfg.k;
+  int nref = 0;
+  for (uint32_t v = v0 + lane; v < v1; v += 32) {
+    int dig[kTileMaxG];
+    uint32_t x = v;
+    for (int b = k - 1; b >= 0; b--) {
+      dig[b] = (int)(x % (uint32_t)L);
+      x /= (uint32_t)L;
+    }
+    float T = 0.f, E = 0.f;
+    for (int b = 0; b < k; b++) {
+      T = fmaxf(T, wp.gt[b * 4 + dig[b]]);
+      E += wp.ge[b * 4 + dig[b]];
+    }
+    unsigned hitm = 0;
+    if constexpr (WS::RT) {
+      hitm = rt_screen<WS>(p, thr, thr_sm, T, E);
+    } else if constexpr (WS::N > 0) {
+      float q[WS::N];
+      WS::q(T, E, q);
+#pragma unroll
+      for (int s = 0; s < WS::N; s++)
+        if (q[s] <= thr.vm[s]) hitm |= 1u << s;
+    }
+    bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(T, p.tlb_scale_f), E);
+    double T64 = 0.0;
+    if (hitm || par) {
+      for (int b = 0; b < k; b++) T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
+      if (par && !hitm) par = !stair_dominated(stair, p, T64, E);
+    }
+    if (hitm || par) {
+      nref += check_config<WS>(tb, *p.gp, stair, wp, thr_sm, lb, wp.base + v, dig, T, E, T64);
+      thr_from_sm<WS>(p, thr, thr_sm);
+    }
+  }
+  return nref;
+}
+
 // All level vectors v in [v0, v1) of the current partition (L = 4).
 // k >= 5: lane = (h, digit of group k-5, digit of group k-4); the warp loop
 // runs over j = digit strings of groups 0..k-6, two per step (h selects);
 // each lane scores the 64-configuration tile of groups k-3..k-1 in registers.
-template <class WS>
+template <int L, class WS>
 __device__ __forceinline__ int partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
                                                  WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
                                                  uint32_t v0, uint32_t v1, int lane) {
+  if constexpr (L != 4) return small_l_configs<L, WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
   const int k = wp.cfg.k;
   if (k < 5) {
     const int r = edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
@@ -728,10 +778,10 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
       if (lane < k * L) {
         const int b = lane / L, mu = lane % L;
         const GroupRec r = gtab[(size_t)wp.cfg.mask[b] * L + mu];
-        wp.gt[b * L + mu] = r.t32;
-        wp.ge[b * L + mu] = r.e32;
-        wp.g64[b * L + mu] = r.t64;
-        wp.ge64[b * L + mu] = r.e64;
+        wp.gt[b * 4 + mu] = r.t32;
+        wp.ge[b * 4 + mu] = r.e32;
+        wp.g64[b * 4 + mu] = r.t64;
+        wp.ge64[b * 4 + mu] = r.e64;
         infeas = r.t32 == __int_as_float(0x7f800000);
       }
       const bool feas = __ballot_sync(0xffffffffu, infeas) == 0u;
@@ -740,7 +790,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
         if (feas) wp.nfeas += v1 - v0;
       }
       __syncwarp();
-      if (feas) nref += partition_configs<WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
+      if (feas) nref += partition_configs<L, WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
       __syncwarp();
       if (base + Pn >= e) break;
       if (lane == 0) {

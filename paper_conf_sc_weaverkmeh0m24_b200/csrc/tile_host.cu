@@ -25,6 +25,13 @@ static bool ws_match(const DevParams &dp, int *perm) {
 
 template <int L>
 static const void *tile_pick_ws(DevParams *dp) {
+  if constexpr (L != 4) {  // 2 or 3 levels: per-configuration path, Pareto-only or run-time weights
+    if (dp->dump) return nullptr;
+    if (dp->nw == 0) return dp->want_pareto ? tile_fn<L, WS_P>() : nullptr;
+    if (dp->nw > kMaxW) return nullptr;
+    for (int s = 0; s < dp->nw; s++) dp->ws_perm[s] = s;
+    return tile_fn<L, WS_RT>();
+  }
   int perm[kMaxW];
   if (dp->dump) {  // sched_debug_scores32: the (1,1) kernel that also dumps every configuration's fp32 score
     if (dp->nw != 1 || dp->wa[0] != 1 || dp->wb[0] != 1) return nullptr;
@@ -64,11 +71,11 @@ size_t tile_smem_bytes(const DevParams &dp) {
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
   const char *b0 = std::getenv("SCHED_B0");
   dp.b0mode = b0 && *b0 ? std::atoi(b0) : 2;  // tile-level only: the partition-level pass costs more than it saves (c4 (1,0): 740 vs 779 ms)
-  if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L != 4 || !dp.gtab_ok) return false;
+  if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L < 2 || dp.L > 4 || !dp.gtab_ok) return false;
   // E = sum_g E_g with level-independent feasibility: COUNT_IDLE (global
   // energy term) and NO_INTERFERENCE (level-dependent feasibility) take the generic kernel
   if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE)) return false;
-  const void *fn = tile_pick_ws<4>(&dp);
+  const void *fn = dp.L == 4 ? tile_pick_ws<4>(&dp) : (dp.L == 3 ? tile_pick_ws<3>(&dp) : tile_pick_ws<2>(&dp));
   if (!fn) return false;
   tl->fn = fn;
   tl->smem = tile_smem_bytes(dp);

@@ -30,10 +30,12 @@ ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--sigma", type=int, default=5)
 ap.add_argument("--slices", type=int, default=64)
 ap.add_argument("--scope", type=int, default=None)
+ap.add_argument("--levels", default=None, help="comma-separated MPS levels, e.g. 50,75,100")
 a = ap.parse_args()
 prof, q = config(a.name)
-if a.scope is not None:
-    q = Query(q.n, q.g, q.c, q.levels, a.scope, q.weights, q.want_pareto)
+if a.scope is not None or a.levels:
+    lv = tuple(int(x) for x in a.levels.split(",")) if a.levels else q.levels
+    q = Query(q.n, q.g, q.c, lv, q.scope if a.scope is None else a.scope, q.weights, q.want_pareto)
 sch = S.Scheduler(prof)
 for s in a.sets.split(","):
     qs = q if SETS[s] is None else Query(q.n, q.g, q.c, q.levels, q.scope, SETS[s], q.want_pareto)
