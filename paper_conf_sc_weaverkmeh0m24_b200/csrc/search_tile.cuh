@@ -414,20 +414,19 @@ __device__ __forceinline__ unsigned rt_screen(const DevParams &p, const Thr<WS> 
   return hit;
 }
 
-// L = 2 or 3 searched levels (any partition) -- the L = 4 tile shape (64
-// configurations of the last three groups in registers, lanes over two more
-// digits) does not apply: every lane takes configurations v0 + lane + 32 i,
-// decodes their base-L level digits and scores them from the partition's
-// group records (T = max, E = sum in block order), screens them (run-time
-// weights: the log-domain pre-screen; Pareto: the fp32 staircase, then the
-// exact fp64 makespan), and sends the rare survivors to check_config.
+// L = 2 or 3 searched levels, per configuration: configurations v of
+// [v0, v1) with stride `step`, decoded into base-L level digits and scored
+// from the partition's group records (T = max, E = block-order sum), screened
+// (run-time weights: log-domain pre-screen; Pareto: fp32 staircase, then the
+// exact fp64 makespan), survivors through check_config.  Used for partitions
+// of fewer than 3 groups and for tiles straddling the unit's range.
 template <int L, class WS>
-__device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                               const WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
-                                               uint32_t v0, uint32_t v1, int lane) {
+__device__ __noinline__ int small_l_edge(const Tables &tb, const DevParams &p, const Stair &stair,
+                                         const WarpPart &wp, float *thr_sm, BestRec *lb, uint32_t v0,
+                                         uint32_t v1, uint32_t step) {
   const int k = wp.cfg.k;
   int nref = 0;
-  for (uint32_t v = v0 + lane; v < v1; v += 32) {
+  for (uint32_t v = v0; v < v1; v += step) {
     int dig[kTileMaxG];
     uint32_t x = v;
     for (int b = k - 1; b >= 0; b--) {
@@ -435,29 +434,113 @@ __device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams
       x /= (uint32_t)L;
     }
     float T = 0.f, E = 0.f;
+    double T64 = 0.0;
     for (int b = 0; b < k; b++) {
       T = fmaxf(T, wp.gt[b * 4 + dig[b]]);
       E += wp.ge[b * 4 + dig[b]];
+      T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
-    unsigned hitm = 0;
-    if constexpr (WS::RT) {
-      hitm = rt_screen<WS>(p, thr, thr_sm, T, E);
-    } else if constexpr (WS::N > 0) {
-      float q[WS::N];
-      WS::q(T, E, q);
+    nref += check_config<WS>(tb, p, stair, wp, thr_sm, lb, wp.base + v, dig, T, E, T64);
+  }
+  return nref;
+}
+
+// L = 2 or 3 searched levels: tiles of the last two groups (L^2
+// configurations, their 2 x L records in registers); every lane takes a
+// contiguous range of the other groups' digit strings ("outer" strings,
+// odometer in base L), per string folds the outer groups into (T_p, E_p),
+// scores the tile's configurations (T = max, E = add, min-reduced to the
+// tile's exact lower corner like the L = 4 tile), screens the corner once and
+// re-checks a tile that is not cleared configuration by configuration.
+template <int L, class WS>
+__device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams &p, const Stair &stair,
+                                               const WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
+                                               uint32_t v0, uint32_t v1, int lane) {
+  const int k = wp.cfg.k;
+  if (k < 3) {
+    const int r = small_l_edge<L, WS>(tb, *p.gp, stair, wp, thr_sm, lb, v0 + lane, v1, 32);
+    thr_from_sm<WS>(p, thr, thr_sm);
+    return r;
+  }
+  constexpr uint32_t TL = (uint32_t)(L * L);
+  const int nb = (k - 2) * 4, nc = (k - 1) * 4;
+  float Bt[L], Be[L], Ct[L], Ce[L];
 #pragma unroll
-      for (int s = 0; s < WS::N; s++)
-        if (q[s] <= thr.vm[s]) hitm |= 1u << s;
+  for (int m = 0; m < L; m++) {
+    Bt[m] = wp.gt[nb + m];
+    Be[m] = wp.ge[nb + m];
+    Ct[m] = wp.gt[nc + m];
+    Ce[m] = wp.ge[nc + m];
+  }
+  double minBC64 = 0.0;
+  {
+    double mb = wp.g64[nb], mc = wp.g64[nc];
+#pragma unroll
+    for (int m = 1; m < L; m++) {
+      mb = fmin(mb, wp.g64[nb + m]);
+      mc = fmin(mc, wp.g64[nc + m]);
     }
-    bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(T, p.tlb_scale_f), E);
-    double T64 = 0.0;
-    if (hitm || par) {
-      for (int b = 0; b < k; b++) T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
-      if (par && !hitm) par = !stair_dominated(stair, p, T64, E);
+    minBC64 = fmax(mb, mc);
+  }
+  // outer strings meeting [v0, v1), split into 32 contiguous lane ranges
+  const uint32_t o_lo = v0 / TL, o_hi = (v1 + TL - 1) / TL;
+  const uint32_t q = (o_hi - o_lo + 31) / 32;
+  uint32_t o = o_lo + min((uint32_t)lane * q, o_hi - o_lo);
+  const uint32_t oe = o_lo + min((uint32_t)(lane + 1) * q, o_hi - o_lo);
+  int dig[kTileMaxG];
+  {
+    uint32_t x = o;
+    for (int b = k - 3; b >= 0; b--) {
+      dig[b] = (int)(x % (uint32_t)L);
+      x /= (uint32_t)L;
     }
-    if (hitm || par) {
-      nref += check_config<WS>(tb, *p.gp, stair, wp, thr_sm, lb, wp.base + v, dig, T, E, T64);
+  }
+  int nref = 0;
+  for (; o < oe; o++) {
+    float Tp = 0.f, Ep = 0.f;
+    for (int b = 0; b < k - 2; b++) {
+      Tp = fmaxf(Tp, wp.gt[b * 4 + dig[b]]);
+      Ep += wp.ge[b * 4 + dig[b]];
+    }
+    const uint32_t vt = o * TL;
+    if (vt < v0 || vt + TL > v1) {  // a tile straddling the unit's range
+      nref += small_l_edge<L, WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + TL < v1 ? vt + TL : v1, 1);
       thr_from_sm<WS>(p, thr, thr_sm);
+    } else {
+      float mT = __int_as_float(0x7f800000), mE = mT;
+#pragma unroll
+      for (int b = 0; b < L; b++) {
+        const float T1 = fmaxf(Tp, Bt[b]), E1 = Ep + Be[b];
+#pragma unroll
+        for (int c = 0; c < L; c++) {
+          mT = fminf(mT, fmaxf(T1, Ct[c]));
+          mE = fminf(mE, E1 + Ce[c]);
+        }
+      }
+      unsigned hitm = 0;
+      if constexpr (WS::RT) {
+        hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
+      } else if constexpr (WS::N > 0) {
+        float mq[WS::N];
+        WS::q(mT, mE, mq);
+#pragma unroll
+        for (int s2 = 0; s2 < WS::N; s2++)
+          if (mq[s2] <= thr.vm[s2]) hitm |= 1u << s2;
+      }
+      bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+      if (par && !hitm) {  // the tile's exact corner makespan
+        double c = minBC64;
+        for (int b = 0; b < k - 2; b++) c = fmax(c, wp.g64[b * 4 + dig[b]]);
+        par = !stair_dominated(stair, p, c, mE);
+      }
+      if (hitm || par) {
+        nref += small_l_edge<L, WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, vt + TL, 1);
+        thr_from_sm<WS>(p, thr, thr_sm);
+      }
+    }
+    for (int b = k - 3; b >= 0; b--) {  // next outer string
+      if (++dig[b] < L) break;
+      dig[b] = 0;
     }
   }
   return nref;
