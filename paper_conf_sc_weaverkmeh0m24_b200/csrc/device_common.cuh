@@ -461,10 +461,24 @@ __device__ __forceinline__ bool group_eval(const Tables &tb, const DevParams &p,
     if (tc > Tg64) Tg64 = tc;
   }
   t32 = Tg;
-  e32 = p.phat * Tg + D;
   t64 = Tg64;
-  e64 = __dadd_rn(__dmul_rn(p.ps, Tg64), D64);
+  if (p.model & SCHED_MODEL_COUNT_IDLE) {
+    // R26: E = G P_s T + sum_g D_g -- the record carries D_g only; the tile
+    // kernel adds kidle * T (fp32) / gps * T (fp64) per configuration
+    e32 = D;
+    e64 = D64;
+  } else {
+    e32 = p.phat * Tg + D;
+    e64 = __dadd_rn(__dmul_rn(p.ps, Tg64), D64);
+  }
   return true;
+}
+
+// a configuration's fp32 E-hat from its T-hat and the sum of its group
+// records' e32 (COUNT_IDLE: the records hold D-hat, R26: E = kidle T + D;
+// monotone in both arguments, so min-reduced corners stay exact bounds)
+__device__ __forceinline__ float e_total(const DevParams &p, float T, float esum) {
+  return (p.model & SCHED_MODEL_COUNT_IDLE) ? fmaf(p.kidle, T, esum) : esum;
 }
 
 // ------------------------------------------------------------ DP walk (RGS state)

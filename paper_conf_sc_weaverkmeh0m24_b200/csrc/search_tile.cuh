@@ -268,6 +268,7 @@ __device__ __noinline__ int check_config(const Tables &tb, const DevParams &p, c
   const double T64r = T64;
   double E64 = 0.0;
   for (int b = 0; b < wp.cfg.k; b++) E64 = __dadd_rn(E64, wp.ge64[b * 4 + dig[b]]);
+  if (p.model & SCHED_MODEL_COUNT_IDLE) E64 = __dadd_rn(__dmul_rn(p.gps, T64r), E64);  // R26 (records: D_g)
   if constexpr (WS::N > 0) {
 #pragma unroll
     for (int s = 0; s < WS::N; s++) {
@@ -312,6 +313,7 @@ __device__ __noinline__ int edge_configs(const Tables &tb, const DevParams &p, c
       E += wp.ge[b * 4 + dig[b]];
       T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
+    E = e_total(p, T, E);
     dump_score<WS>(p, wp.base + v, T, E);
     if constexpr (WS::RT) {
       for (int s = 0; s < p.nw; s++) thr[s] = fminf(thr[s], rt_q(p, s, T, E));
@@ -346,16 +348,17 @@ __device__ __noinline__ int tile_slow(const Tables &tb, const DevParams &p, cons
   const float minCe = fminf(fminf(wp.ge[gc], wp.ge[gc + 1]), fminf(wp.ge[gc + 2], wp.ge[gc + 3]));
   const float minBe = fminf(fminf(wp.ge[gb], wp.ge[gb + 1]), fminf(wp.ge[gb + 2], wp.ge[gb + 3]));
   int nref = 0;
+  const bool prune = !arg_hit && !(p.model & SCHED_MODEL_COUNT_IDLE);  // idle: corner E needs T (not tracked here)
   for (int a = 0; a < 4; a++) {
     const float T1 = fmaxf(Tp, wp.gt[ga + a]), E1 = Ep + wp.ge[ga + a];
     const double A64 = fmax(Tp64, wp.g64[ga + a]);
-    if (!arg_hit && stair_dominated(stair, p, fmax(fmax(A64, minB64), minC64), (E1 + minBe) + minCe)) continue;
+    if (prune && stair_dominated(stair, p, fmax(fmax(A64, minB64), minC64), (E1 + minBe) + minCe)) continue;
     for (int b = 0; b < 4; b++) {
       const float T2 = fmaxf(T1, wp.gt[gb + b]), E2 = E1 + wp.ge[gb + b];
       const double B64 = fmax(A64, wp.g64[gb + b]);
-      if (!arg_hit && stair_dominated(stair, p, fmax(B64, minC64), E2 + minCe)) continue;
+      if (prune && stair_dominated(stair, p, fmax(B64, minC64), E2 + minCe)) continue;
       for (int c = 0; c < 4; c++) {
-        const float T = fmaxf(T2, wp.gt[gc + c]), E = E2 + wp.ge[gc + c];
+        const float T = fmaxf(T2, wp.gt[gc + c]), E = e_total(p, T, E2 + wp.ge[gc + c]);
         const double T64 = fmax(B64, wp.g64[gc + c]);
         dig[k - 3] = a;
         dig[k - 2] = b;
@@ -440,6 +443,7 @@ __device__ __noinline__ int small_l_edge(const Tables &tb, const DevParams &p, c
       E += wp.ge[b * 4 + dig[b]];
       T64 = fmax(T64, wp.g64[b * 4 + dig[b]]);
     }
+    E = e_total(p, T, E);
     nref += check_config<WS>(tb, p, stair, wp, thr_sm, lb, wp.base + v, dig, T, E, T64);
   }
   return nref;
@@ -517,6 +521,7 @@ __device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams
           mE = fminf(mE, E1 + Ce[c]);
         }
       }
+      mE = e_total(p, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D)
       unsigned hitm = 0;
       if constexpr (WS::RT) {
         hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
@@ -643,10 +648,11 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
               const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
-              dump_score<WS>(p, wp.base + vt + (uint32_t)(a * 16 + b * 4 + c), T, E);
+              dump_score<WS>(p, wp.base + vt + (uint32_t)(a * 16 + b * 4 + c), T, e_total(p, T, E));
             }
           }
         }
+        mE = e_total(p, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D)
         if constexpr (WS::RT) {
           hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
         } else {
@@ -671,6 +677,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
           }
         }
+        cE = e_total(p, cT, cE);
       }
       hitm &= ~b0skip;
       double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
@@ -728,6 +735,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             }
           }
         }
+        mE = e_total(p, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D)
         if constexpr (WS::RT) {
           hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
         } else {
@@ -752,6 +760,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
           }
         }
+        cE = e_total(p, cT, cE);
       }
       hitm = full ? (hitm & ~b0skip) : 0u;
       // exact tile corner (fp64 min makespan) where a screen needs it: b = 0

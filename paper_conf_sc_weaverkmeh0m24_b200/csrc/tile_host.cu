@@ -74,7 +74,7 @@ bool tile_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.scope != SCHED_PER_GPU || dp.g > kTileMaxG || dp.L < 2 || dp.L > 4 || !dp.gtab_ok) return false;
   // E = sum_g E_g with level-independent feasibility: COUNT_IDLE (global
   // energy term) and NO_INTERFERENCE (level-dependent feasibility) take the generic kernel
-  if (dp.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_NO_INTERFERENCE)) return false;
+  if (dp.model & SCHED_MODEL_NO_INTERFERENCE) return false;  // level-dependent feasibility: generic kernel
   const void *fn = dp.L == 4 ? tile_pick_ws<4>(&dp) : (dp.L == 3 ? tile_pick_ws<3>(&dp) : tile_pick_ws<2>(&dp));
   if (!fn) return false;
   tl->fn = fn;

@@ -77,3 +77,28 @@ def test_variants_big_windows(name, model):
     for lo in [0, tot - 50_000] + [rnd.randrange(tot - 50_000) for _ in range(2)]:
         qw = q.with_range(lo, lo + 50_000)
         check(sch.search(qw), oracle.search(prof, qw), qw)
+
+
+@pytest.mark.parametrize("model", [1, 5, 9, 13])
+@pytest.mark.parametrize("levels", [(25, 50, 75, 100), (50, 75, 100)])
+def test_count_idle_tile_kernel(model, levels):
+    """COUNT_IDLE (R26: every GPU draws P_s for the whole makespan, E = G P_s T
+    + sum D_g) and its combinations with POWER_CAP / TIME_SLICE on the PER_GPU
+    tile kernel (round 2: the group records carry D_g, the kernel adds the
+    idle term per configuration and to every tile corner): small full spaces
+    and c4 windows, bitwise against the oracle."""
+    prof = make_profile(9, levels=(25, 50, 75, 100), seed=43)
+    q = Query(9, 6, 4, levels, PER_GPU, ((1, 1), (2, 1), (1, 0), (0, 1)), True, model=model, power_cap=130.0)
+    res = S.Scheduler(prof).search(q)
+    assert res.stats["kernel_path"] == 1
+    check(res, oracle.search(prof, q), q)
+    prof4, q4 = config("c4")
+    q4 = dataclasses.replace(q4, levels=levels, model=model, power_cap=300.0)
+    tot = S.count(q4)
+    sch = S.Scheduler(prof4)
+    rnd = random.Random(model)
+    for lo in [0, tot - 100_000, (1 << 24) - 50_000] + [rnd.randrange(tot - 100_000) for _ in range(2)]:
+        qw = q4.with_range(lo, lo + 100_000)
+        r = sch.search(qw)
+        assert r.stats["kernel_path"] == 1
+        check(r, oracle.search(prof4, qw), qw)
