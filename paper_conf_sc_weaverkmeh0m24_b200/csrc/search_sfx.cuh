@@ -37,7 +37,13 @@
 
 namespace sched {
 
-constexpr int kSfxThreads = 256;
+#ifndef SCHED_SFX_THREADS
+#define SCHED_SFX_THREADS 256
+#endif
+#ifndef SCHED_SFX_MINB
+#define SCHED_SFX_MINB 2
+#endif
+constexpr int kSfxThreads = SCHED_SFX_THREADS;
 constexpr int kSfxWarps = kSfxThreads / 32;
 constexpr int kSfxMaxG = 8;
 
@@ -473,7 +479,7 @@ __device__ __forceinline__ float2 sfx_entry(const DevParams &p, const GroupRec *
 }
 
 template <int M>
-__global__ void __launch_bounds__(kSfxThreads, 2) k_sfx(const DevParams p) {
+__global__ void __launch_bounds__(kSfxThreads, SCHED_SFX_MINB) k_sfx(const DevParams p) {
   extern __shared__ __align__(16) unsigned char sm[];
   stage_blob(sm, p);
   const Tables tb = tables_at(sm, p);
