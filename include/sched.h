@@ -268,8 +268,9 @@ int sched_score(const sched_handle *h, const sched_query *q, uint64_t index, int
  * vectors, then the block-order DP over workflow subsets.  Reaches spaces
  * that cannot be enumerated, e.g. the literal per-client c4 (16 workflows,
  * 8 GPUs, 4 levels per client: 4.05e19 configurations).  Requires
- * 2 <= n <= 20, L^max_clients <= 2^32 (PER_CLIENT), no SCHED_MODEL_COUNT_IDLE
- * or SCHED_MODEL_TIME_SLICE;
+ * 2 <= n <= 20, L^max_clients <= 2^32 (PER_CLIENT), no SCHED_MODEL_TIME_SLICE
+ * (SCHED_MODEL_COUNT_IDLE: the DP adds up the dynamic energies and applies
+ * the idle term G P_s T to the whole-set front);
  * the index window and shard fields must be the defaults (whole space, one
  * shard).  front[front_cap] is ordered by X descending (T ascending), one
  * witness configuration per distinct (T, E); best[W] is the max F_w over the

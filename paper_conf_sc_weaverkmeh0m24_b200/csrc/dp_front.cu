@@ -92,6 +92,14 @@ __device__ __forceinline__ bool front_insert(P *f, int &n, const P &x) {
 
 // exact canonical fp64 (T_B, E_B) of group B with per-member level digits
 // lev[i] (digit of workflow i); false if infeasible (R27)
+// the group term the DP adds up: E_g = P_s T_g + D_g (canonical), or D_g
+// alone under COUNT_IDLE (R26: E = G P_s T + sum_g D_g; k_dp_final adds the
+// idle term to the whole-set front, E is monotone in (T, sum D), so the
+// (T, sum D) front holds every (T, E) front point)
+__device__ __forceinline__ double dp_eg(const DevParams &p, double Tg, double D) {
+  return (p.model & SCHED_MODEL_COUNT_IDLE) ? D : __dadd_rn(__dmul_rn(p.ps, Tg), D);
+}
+
 __device__ __forceinline__ bool group64(const Tables &tb, const DevParams &p, uint32_t B, const int *lev,
                                         double &Tout, double &Eout) {
   const double ps = p.ps;
@@ -126,7 +134,7 @@ __device__ __forceinline__ bool group64(const Tables &tb, const DevParams &p, ui
     if (tcap > Tg) Tg = tcap;
   }
   Tout = Tg;
-  Eout = __dadd_rn(__dmul_rn(ps, Tg), D);
+  Eout = dp_eg(p, Tg, D);
   return true;
 }
 
@@ -358,7 +366,7 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
           const double tcap = __ddiv_rn(Dmin, p.capd);
           if (tcap > Tmin) Tmin = tcap;
         }
-        const double Emin = __dadd_rn(__dmul_rn(ps, Tmin), Dmin);
+        const double Emin = dp_eg(p, Tmin, Dmin);
         bool skip = wt <= Tmin && we <= Emin;
         for (int i = 0; i < nf && !skip; i++)
           if (f[i].t <= Tmin && f[i].e <= Emin) {
@@ -413,7 +421,7 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
             }
             PPt x;
             x.t = Tg;
-            x.e = __dadd_rn(__dmul_rn(ps, Tg), Dl);
+            x.e = dp_eg(p, Tg, Dl);
             x.v = (uint32_t)(base + (uint32_t)((d0 * L + d1) * L + d2));
             x.pad = 0;
             // quick reject: a point inserted earlier (lt, le) dominates or equals x ->
@@ -480,7 +488,7 @@ __device__ __forceinline__ void pf_split(const A &tb, const DevParams &p, uint32
       }
       PPt x;
       x.t = Tg;
-      x.e = __dadd_rn(__dmul_rn(ps, Tg), Dl);
+      x.e = dp_eg(p, Tg, Dl);
       x.v = (uint32_t)(base + lv);
       x.pad = 0;
       ok &= front_insert<kLF>(f, nf, x);
@@ -794,6 +802,15 @@ __global__ void k_dp_final(const DpParams dp, DpOut *out, int cap, int *nout, in
   if (threadIdx.x || blockIdx.x) return;
   const int G = dp.p.g;
   const uint32_t full = dp.n >= 32 ? 0xffffffffu : (1u << dp.n) - 1;
+  if (dp.p.model & SCHED_MODEL_COUNT_IDLE) {  // R26: E = (G P_s) T + sum_g D_g (group order), as the oracle
+    for (int k = 1; k <= G; k++) {
+      const size_t st = (size_t)(full >> 1) * (G + 1) + k;
+      for (int i = 0; i < dp.frcnt[st]; i++) {
+        DPt &x = dp.fr[st * kFM + i];
+        x.e = __dadd_rn(__dmul_rn(dp.p.gps, x.t), x.e);
+      }
+    }
+  }
   int n = 0;
   for (int k = 1; k <= G; k++) {
     const size_t st = (size_t)(full >> 1) * (G + 1) + k;
@@ -919,7 +936,7 @@ void dp_groups(const Profile &P, const Query &q, std::vector<uint32_t> *smask, s
 }  // namespace
 
 int dp_front_workspace(const Profile &P, const Query &q, const DevParams &dp, size_t *bytes) {
-  if (q.n < 2 || q.n > 20 || q.g > kMaxG || (q.model & (SCHED_MODEL_COUNT_IDLE | SCHED_MODEL_TIME_SLICE)))
+  if (q.n < 2 || q.n > 20 || q.g > kMaxG || (q.model & SCHED_MODEL_TIME_SLICE))
     return SCHED_E_INVALID;
   if (q.scope == SCHED_PER_CLIENT) {
     double lg = 0.0;  // L^C must fit the 32-bit vector id

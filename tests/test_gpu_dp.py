@@ -176,3 +176,25 @@ def test_dp_front_c4_literal_per_client_no_better_neighbour_or_sample():
         lab = [rnd.randrange(G) for _ in range(n)]
         nfeas += check(_canon(lab), [rnd.randrange(L) for _ in range(n)])
     assert nfeas > 10000
+
+
+@pytest.mark.parametrize("model", [1, 5])
+@pytest.mark.parametrize("n,g,c,levels,scope,seed", [
+    (6, 3, 3, (50, 100), PER_CLIENT, 711), (7, 3, 7, (25, 50, 75, 100), PER_CLIENT, 712),
+    (9, 4, 4, (25, 50, 75, 100), PER_GPU, 713), (8, 8, 8, (100,), PER_GPU, 714),
+])
+def test_dp_front_count_idle_vs_enumeration(model, n, g, c, levels, scope, seed):
+    """COUNT_IDLE (R26: E = G P_s T + sum D_g; round 2: the DP adds up D_g and
+    applies the idle term to the whole-set front) alone and with POWER_CAP:
+    front values, per-weight optimum and witnesses equal the oracle's full
+    enumeration."""
+    prof = make_profile(n, levels=(25, 50, 75, 100), seed=seed)
+    q = Query(n, g, c, levels, scope, W, True, model=model, power_cap=140.0)
+    ref = oracle.search(prof, q)
+    rc, best, front, st = S.Scheduler(prof).front_dp(q)
+    assert st["kernel_path"] == 4
+    assert [(p.makespan_s, p.energy_j) for p in front] == [(T, E) for _, T, E in ref["pareto"]]
+    for w in range(len(W)):
+        assert best[w].score64 == ref["best"][w][1]
+    for p in list(front) + list(best):
+        assert _witness_ok(prof, q, p)
