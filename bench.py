@@ -180,9 +180,9 @@ def check_steps(step_cfg, first_sigma, space, world, dev):
     the index count of that step's slice (dist.check_coverage raises)."""
     import torch
     from paper_conf_sc_weaverkmeh0m24_b200.dist import check_coverage
+    import torch.distributed as dist
     t = torch.tensor(step_cfg, dtype=torch.int64, device=dev)
-    if world > 1:
-        import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized():
         dist.all_reduce(t)
     for i, n in enumerate(t.tolist()):
         check_coverage(n, 0, space, CHUNK_LOG2, (first_sigma + i) % SLICES, SLICES, world)
@@ -295,13 +295,16 @@ def run_ours(args):
     from synth import config
 
     rank, world, local = env()
+    # a process group whenever the launcher is torchrun (also at one rank:
+    # `torchrun --nproc-per-node 1` exercises the NCCL exchange on one GPU)
+    pg = world > 1 or "TORCHELASTIC_RUN_ID" in os.environ
     assert torch.cuda.is_available(), "bench.py needs a CUDA device"
     # BENCH_SHARE_GPU=1 (tests only): every rank uses cuda:0 with a gloo group,
     # to exercise the N > 1 path on a one-GPU box; NCCL otherwise.
     share = os.environ.get("BENCH_SHARE_GPU") == "1"
     local = 0 if share else local
     torch.cuda.set_device(local)
-    if world > 1:
+    if pg:
         if share:
             dist.init_process_group("gloo")
         else:
@@ -317,14 +320,14 @@ def run_ours(args):
 
     def barrier():
         torch.cuda.synchronize()
-        if world > 1:
+        if pg:
             dist.barrier()
         torch.cuda.synchronize()
 
     def step(sigma, sch=sched, workspace=ws):
         res = sch.search(q, workspace=workspace, shard=((sigma % SLICES) * world + rank, SLICES * world),
                          chunk_log2=CHUNK_LOG2)
-        if world > 1:
+        if pg:
             best, par, _ = exchange(res.best, res.pareto, nw)
         else:
             best, par = res.best, res.pareto
@@ -362,7 +365,7 @@ def run_ours(args):
     clk = clocks.stop()
     elapsed = ev0.elapsed_time(ev1)
     rdev = "cpu" if share else "cuda"
-    if world > 1:
+    if pg:
         t = torch.tensor([elapsed, float(ncfg)], dtype=torch.float64, device=rdev)
         mx = t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
@@ -389,7 +392,7 @@ def run_ours(args):
         fresh.close()
     barrier()
     e_dt = time.perf_counter() - t0
-    if world > 1:
+    if pg:
         t = torch.tensor([e_dt, float(e_cfg)], dtype=torch.float64, device=rdev)
         mx = t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
@@ -401,7 +404,7 @@ def run_ours(args):
                    "kernels, D2H of counters/picks, NCCL exchange + merge; host wall clock"}
 
     if rank != 0:
-        dist.destroy_process_group() if world > 1 else None
+        dist.destroy_process_group() if pg else None
         return 0
     # time-to-optimal-schedule of the same space by the device subset DP
     # (sched_front_dp): exact front + optimum per weight.
@@ -462,7 +465,7 @@ def run_ours(args):
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(prof, q)
     print(json.dumps(line), flush=True)
-    if world > 1:
+    if pg:
         dist.destroy_process_group()
     return 0
 
@@ -489,6 +492,9 @@ def run_full(args, step, barrier, rank, world, space, nw):
                           "configs_per_s": space / dt,
                           "best": [(b.index, b.score64) for b in mb],
                           "pareto": [(p.index, p.makespan_s, p.energy_j) for p in mp]}), flush=True)
+    import torch.distributed as dist
+    if dist.is_initialized():
+        dist.destroy_process_group()
     return 0
 
 

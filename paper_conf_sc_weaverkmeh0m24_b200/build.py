@@ -14,8 +14,11 @@ from concurrent.futures import ThreadPoolExecutor
 HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
-OBJ = os.path.join(HERE, "build_obj")
-SO = os.path.join(HERE, "libsched.so")
+# SCHED_BUILD_TAG=X (A/B measurements): objects in build_obj_X/, library ab/lib_X.so
+# (load it with SCHED_SO_PATH=ab/lib_X.so); the product build leaves it unset
+_TAG = os.environ.get("SCHED_BUILD_TAG", "")
+OBJ = os.path.join(HERE, "build_obj" + ("_" + _TAG if _TAG else ""))
+SO = os.path.join(ROOT, "ab", f"lib_{_TAG}.so") if _TAG else os.path.join(HERE, "libsched.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -51,6 +54,7 @@ def _compile(src):
 
 def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(OBJ, exist_ok=True)
+    os.makedirs(os.path.dirname(SO), exist_ok=True)
     hdr = _newest_header()
     todo = [s for s in sources()
             if force or not os.path.exists(_obj(s))

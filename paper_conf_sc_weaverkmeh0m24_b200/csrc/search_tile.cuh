@@ -101,14 +101,21 @@ struct WS_SWEEP {  // c5 sweep (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
 // corner screen evaluates q_w = T^a E^b by repeated multiplication; the
 // lane's running thresholds live in its shared-memory row (thr_sm), not in
 // registers, so the tile loop's register footprint is that of WS_11_21.
-struct WS_RT {
-  static constexpr int N = kMaxW;
+template <int NW, bool B0>
+struct WS_RTT {
+  static constexpr int N = NW;         // weight slots (the query's p.nw <= NW are used)
   static constexpr bool RT = true;
+  static constexpr bool MAYB0 = B0;    // the set may hold b = 0 weights (vote-guarded tile loop)
   static constexpr bool DUMP = false;
   __host__ __device__ static constexpr int A(int) { return 0; }
   __host__ __device__ static constexpr int B(int) { return 0; }
   __device__ static __forceinline__ void q(float, float, float *) {}
 };
+struct WS_RT : WS_RTT<kMaxW, true> {};
+// every b >= 1 (host-checked): the plain tile loop, like the compiled sets
+// without b = 0 weights; up to 4 weights with 4 threshold registers
+struct WS_RTN : WS_RTT<kMaxW, false> {};
+struct WS_RT4N : WS_RTT<4, false> {};
 
 // WS_11 that also writes every configuration's fp32 (T-hat, E-hat), as the
 // tile loop computes them, to p.dump (sched_debug_scores32: the hot loop's
@@ -122,6 +129,14 @@ __device__ __forceinline__ void dump_score(const DevParams &p, u64 idx, float T,
   if constexpr (WS::DUMP) {
     if (idx >= p.dump_lo && idx - p.dump_lo < p.dump_n) ((float2 *)p.dump)[idx - p.dump_lo] = make_float2(T, E);
   }
+}
+
+// three-input fp32 max (one FMNMX3, the ALU slot of a two-input max;
+// max is exact, so the value is that of fmaxf(fmaxf(a, b), c))
+__device__ __forceinline__ float fmax3f(float a, float b, float c) {
+  float d;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
 }
 
 // q_s = (T/T_seq)^a (E/E_seq)^b for query weight s, run-time exponents
@@ -195,7 +210,7 @@ __device__ __forceinline__ unsigned b0_beaten(const DevParams &p, const BestRec 
 template <class WS>
 __host__ __device__ constexpr bool ws_has_b0() {
   if constexpr (WS::RT) {
-    return true;
+    return WS::MAYB0;
   } else {
     for (int s = 0; s < WS::N; s++)
       if (WS::B(s) == 0) return true;
@@ -390,7 +405,7 @@ __device__ __forceinline__ void thr_from_sm(const DevParams &p, Thr<WS> &thr, co
     for (int s = 0; s < WS::N; s++) thr.vm[s] = thr_sm[s] * p.mul[p.ws_perm[s]];
   } else {  // log2 thresholds of the pre-screen (rt_screen), +inf while unset
 #pragma unroll
-    for (int s = 0; s < kMaxW; s++)
+    for (int s = 0; s < WS::N; s++)
       if (s < p.nw) thr.vm[s] = __log2f(thr_sm[s] * p.mul[s]) + p.lmargin[s];
   }
 }
@@ -407,7 +422,7 @@ __device__ __forceinline__ unsigned rt_screen(const DevParams &p, const Thr<WS> 
   const bool inr = fabsf(lt) < 32.f && fabsf(le) < 32.f;
   unsigned pre = 0;
 #pragma unroll
-  for (int s = 0; s < kMaxW; s++)
+  for (int s = 0; s < WS::N; s++)
     if (s < p.nw && (!inr || fmaf(p.fa[s], lt, p.fb[s] * le) <= thr.vm[s])) pre |= 1u << s;
   unsigned hit = 0;
   if (pre) {
@@ -642,10 +657,18 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
           const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
   #pragma unroll
           for (int b = 0; b < 4; b++) {
-            const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
+#ifdef SCHED_TILE_T2
+            const float T2 = fmaxf(T1, Bt[b]);
+#endif
+            const float E2 = E1 + Be[b];
   #pragma unroll
             for (int c = 0; c < 4; c++) {
-              const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
+#ifdef SCHED_TILE_T2
+              const float T = fmaxf(T2, Ct[c]);
+#else
+              const float T = fmax3f(T1, Bt[b], Ct[c]);  // one ALU slot per configuration, no per-pair T2
+#endif
+              const float E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
               dump_score<WS>(p, wp.base + vt + (uint32_t)(a * 16 + b * 4 + c), T, e_total(p, T, E));

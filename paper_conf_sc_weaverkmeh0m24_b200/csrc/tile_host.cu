@@ -55,10 +55,16 @@ static const void *tile_pick_ws(DevParams *dp) {
   TRY(WS_C1)      // BASELINE configs[0]'s objectives: (1,0) (0,1) (1,1) (2,1)
   TRY(WS_SWEEP)   // configs[4]'s sweep: (1,0) (3,1) (2,1) (1,1) (1,2) (1,3) (0,1)
 #undef TRY
-  // any other 1 <= W <= 8: run-time exponents (query order)
+  // any other 1 <= W <= 8: run-time exponents (query order); without b = 0
+  // weights the plain tile loop (WS_RTN)
   if (dp->nw >= 1 && dp->nw <= kMaxW) {
-    for (int s = 0; s < dp->nw; s++) dp->ws_perm[s] = s;
-    return tile_fn<L, WS_RT>();
+    bool b0 = false;
+    for (int s = 0; s < dp->nw; s++) {
+      dp->ws_perm[s] = s;
+      b0 |= dp->wb[s] == 0;
+    }
+    if (b0) return tile_fn<L, WS_RT>();
+    return dp->nw <= 4 ? tile_fn<L, WS_RT4N>() : tile_fn<L, WS_RTN>();
   }
   return nullptr;
 }

@@ -17,6 +17,8 @@ struct WS_11_21;
 struct WS_SWEEP;
 struct WS_C1;
 struct WS_RT;
+struct WS_RTN;
+struct WS_RT4N;
 struct WS_11_DUMP;
 
 template <int L, class WS>

@@ -19,7 +19,9 @@ SETS = {
     "c1_set": ((1, 0), (0, 1), (1, 1), (2, 1)),                       # BASELINE configs[0]'s objectives
     "c5_sweep": ((1, 0), (3, 1), (2, 1), (1, 1), (1, 2), (1, 3), (0, 1)),   # configs[4]'s sweep
     "eight": ((1, 0), (0, 1), (1, 1), (2, 1), (1, 2), (3, 1), (1, 3), (4, 4)),
-    "single_12": ((1, 2),),
+    "single_12": ((1, 2),),                                            # WS_RT4N (no b = 0 weight)
+    "rt4n": ((1, 1), (2, 1), (1, 2)),                                  # WS_RT4N
+    "rtn6": ((1, 1), (2, 1), (1, 2), (3, 1), (1, 3), (2, 2)),          # WS_RTN (5..8 weights, every b >= 1)
 }
 
 
