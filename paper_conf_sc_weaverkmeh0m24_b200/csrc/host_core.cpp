@@ -543,6 +543,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->kcap = (q.model & SCHED_MODEL_POWER_CAP) ? (float)(eseq / (dp->capd * tseq)) : 0.f;
   dp->gps = (double)q.g * (double)P.ps;
   dp->kidle = (float)(dp->gps * tseq / eseq);
+  dp->kidle0 = (q.model & SCHED_MODEL_COUNT_IDLE) ? dp->kidle : 0.f;
   dp->mem_cap = P.mem_cap;
   dp->want_pareto = q.want_pareto;
   for (int w = 0; w < q.nw; w++) {
@@ -631,8 +632,7 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
     const double tl = (double)tlow * 0.5 * tseq;
     uint64_t b;
     std::memcpy(&b, &tl, 8);
-    dp->bucket_shift = kBucketShift;
-    dp->bucket_base = (uint32_t)(b >> kBucketShift);
+    set_buckets(*dp, kBucketShift, (uint32_t)(b >> kBucketShift));
   }
   std::memcpy(B + dp->off_W, sp.W.data(), 8 * sp.W.size());
   std::memcpy(B + dp->off_trans, sp.trans.data(), 2 * sp.trans.size());

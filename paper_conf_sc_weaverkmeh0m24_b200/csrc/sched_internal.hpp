@@ -84,10 +84,15 @@ struct DevParams {
   double capd;              // P_cap - P_s (exact) for POWER_CAP
   float kcap;               // E_seq / ((P_cap - P_s) T_seq): normalised capped time = D-hat * kcap
   float kidle;              // g P_s T_seq / E_seq: COUNT_IDLE energy term per normalised T
+  float kidle0;             // kidle under COUNT_IDLE, else 0 (tile loop: E + kidle0 T as one FFMA)
   double gps;               // g * P_s (exact) for COUNT_IDLE
   int mem_cap, want_pareto, root, nstates;
   uint32_t bucket_base;     // (bits64(T_lower) >> bucket_shift)
   int bucket_shift;         // kBucketShift, or finer after the seed pass (re-bucketing, search.cu)
+  // the same buckets from the bits of a float T (stair_dominated_f):
+  // bucket = (bits32(T) >> bkt_sh32) + bkt_off32 (mod 2^32); set_buckets() keeps them in step
+  int bkt_sh32;
+  uint32_t bkt_off32;
   // work split
   uint64_t lo, hi;          // window
   uint64_t first_chunk;     // first owned chunk id
@@ -122,6 +127,15 @@ struct DevParams {
                                // out-of-line slow paths, so no thread copies the kernel parameters
                                // to its stack (local memory)
 };
+// bucket_shift / bucket_base and their float-bits form (bits64(x) >> s ==
+// (bits32(x) >> (s - 29)) + (896 << (52 - s)) for a float x, s >= 29)
+inline void set_buckets(DevParams &dp, int shift, uint32_t base) {
+  dp.bucket_shift = shift;
+  dp.bucket_base = base;
+  dp.bkt_sh32 = shift - 29;
+  dp.bkt_off32 = (896u << (52 - shift)) - base;
+}
+
 
 enum {
   kCtrUnit = 0,      // next work unit

@@ -692,10 +692,8 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
         uint64_t b;
         std::memcpy(&b, &span[0], 8);
         const int64_t base = (int64_t)(b >> sh) - 512;
-        dp_full.bucket_shift = sh;
-        dp_full.bucket_base = (uint32_t)std::max<int64_t>(0, base);
-        dp.bucket_shift = dp_full.bucket_shift;
-        dp.bucket_base = dp_full.bucket_base;
+        set_buckets(dp_full, sh, (uint32_t)std::max<int64_t>(0, base));
+        set_buckets(dp, sh, dp_full.bucket_base);
         keep = span_rerun ? 0 : 3;   // the re-run starts a fresh staircase in the finer buckets
       }
     }

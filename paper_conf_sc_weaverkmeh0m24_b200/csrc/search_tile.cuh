@@ -186,6 +186,35 @@ __device__ __forceinline__ bool stair_dominated_f(const Stair &s, const DevParam
   return false;
 }
 
+// the CTA staircase's pm / bp arrays as shared-window addresses: the tile
+// loop's screen loads them with ld.shared (a generic pointer costs a
+// generic LD per tile)
+struct StairSm {
+  uint32_t pm, bp;
+};
+
+__device__ __forceinline__ StairSm stair_sm(const Stair &s) {
+  return StairSm{(uint32_t)__cvta_generic_to_shared(s.pm), (uint32_t)__cvta_generic_to_shared(s.bp)};
+}
+
+// stair_dominated_f with the bucket from the host-made float-bits constants
+// (p.bkt_sh32, p.bkt_off32) and shared-window loads
+__device__ __forceinline__ bool stair_dominated_fs(const StairSm &s, const DevParams &p, float tlb, float eh) {
+  const int b = (int)((__float_as_uint(tlb) >> p.bkt_sh32) + p.bkt_off32);
+  const uint32_t j = (uint32_t)(b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b));
+  const unsigned int eb = __float_as_uint(eh);
+  unsigned int pm;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(pm) : "r"(s.pm + 4u * j));
+  if (eb > pm) return true;
+  unsigned long long pr;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(pr) : "r"(s.bp + 8u * j));
+  if (eb > (unsigned int)(pr >> 32)) {
+    const CandRec *c = (const CandRec *)p.cand + (unsigned int)pr;
+    return (double)tlb >= __ldcg(&c->t);
+  }
+  return false;
+}
+
 // bit s set: weight s has b = 0 (F = X^a depends on T alone) and the lane's
 // best for it has T <= T64 and a lower index than idx: configurations with
 // makespan >= T64 and index >= idx have F <= that best's F (rounding is
@@ -572,8 +601,8 @@ __device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams
 // each lane scores the 64-configuration tile of groups k-3..k-1 in registers.
 template <int L, class WS>
 __device__ __forceinline__ int partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
-                                                 WarpPart &wp, Thr<WS> &thr, float *thr_sm, BestRec *lb,
-                                                 uint32_t v0, uint32_t v1, int lane) {
+                                                 const StairSm &ss, WarpPart &wp, Thr<WS> &thr, float *thr_sm,
+                                                 BestRec *lb, uint32_t v0, uint32_t v1, int lane) {
   if constexpr (L != 4) return small_l_configs<L, WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
   const int k = wp.cfg.k;
   if (k < 5) {
@@ -592,7 +621,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     wp.lp[j] = make_float2(T, E);
   }
   __syncwarp();
-  const int h = lane >> 4, l4 = lane & 15;
+  const int l4 = lane & 15;
   const int ga = (k - 3) * 4, gb = (k - 2) * 4, gc = (k - 1) * 4;
   const float Tl = fmaxf(wp.gt[(k - 5) * 4 + (l4 >> 2)], wp.gt[(k - 4) * 4 + (l4 & 3)]);
   const float El = wp.ge[(k - 5) * 4 + (l4 >> 2)] + wp.ge[(k - 4) * 4 + (l4 & 3)];
@@ -627,24 +656,33 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
                                                fminf(fminf(Bt[0], Bt[1]), fminf(Bt[2], Bt[3]))),
                                          fminf(fminf(Ct[0], Ct[1]), fminf(Ct[2], Ct[3])));
   int nref = 0;
-  const uint32_t s_lo = v0 >> 11, s_hi = (v1 - 1) >> 11;
   if constexpr (!ws_has_b0<WS>()) {
     // sets without b = 0 weights (the c4 bench set): the plain loop; its rare
     // paths are divergent calls (measured faster here than vote-guarded ones:
-    // c4 slice 639 vs 700 ms)
-    for (uint32_t st = s_lo; st <= s_hi; st++) {
-      const uint32_t j = 2 * st + h;
-      const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
-      if (j >= (uint32_t)nloop || vt + 64 <= v0 || vt >= v1) continue;
-      const float2 lp = wp.lp[j];
+    // c4 slice 639 vs 700 ms).  Tile t (v = 64t .. 64t+63) belongs to lane
+    // t mod 32 (t = 32 step + lane: loop string j = t >> 4, lane digits
+    // t & 15 = l4).  The (at most two) tiles cut by the unit's range are
+    // checked per configuration first; the loop then runs over the lane's
+    // full tiles without bounds checks.
+    const uint32_t tb0 = v0 >> 6, tb1 = (v1 - 1) >> 6;
+    bool edge = false;
+    if ((v0 & 63u) && (tb0 & 31u) == (uint32_t)lane) {
+      nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, v0, min(v1, (tb0 + 1) << 6), 1);
+      edge = true;
+    }
+    if ((v1 & 63u) && (tb1 & 31u) == (uint32_t)lane && !(tb1 == tb0 && (v0 & 63u))) {
+      nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, max(v0, tb1 << 6), v1, 1);
+      edge = true;
+    }
+    if (edge) thr_from_sm<WS>(p, thr, thr_sm);
+    const uint32_t te = v1 >> 6;
+    const uint32_t tf = (v0 + 63u) >> 6;
+    for (uint32_t t = tf + (((uint32_t)lane - tf) & 31u); t < te; t += 32) {
+      const float2 lp = wp.lp[t >> 4];
       const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
-      if (vt < v0 || vt + 64 > v1) {  // partial tile at a unit boundary
-        nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
-        thr_from_sm<WS>(p, thr, thr_sm);
-        continue;
-      }
       unsigned hitm = 0;
       float cE, cT;
+      bool fdom = false;  // WS::RT: corner discarded by the fp32 staircase screen
       if constexpr (WS::N > 0) {
         // every configuration's (T, E), min-reduced over the tile: the tile's
         // exact lower corner.  q_w = T^a E^b is monotone in T and E, so the
@@ -671,13 +709,23 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
               const float E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
-              dump_score<WS>(p, wp.base + vt + (uint32_t)(a * 16 + b * 4 + c), T, e_total(p, T, E));
+              dump_score<WS>(p, wp.base + (t << 6) + (uint32_t)(a * 16 + b * 4 + c), T, e_total(p, T, E));
             }
           }
         }
-        mE = e_total(p, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D)
+        // the exact corner's E: COUNT_IDLE adds kidle T as one FFMA; without
+        // it kidle0 = 0 and fma(0, T, E) == E exactly (T finite: feasible partition)
+        mE = fmaf(p.kidle0, mT, mE);
         if constexpr (WS::RT) {
-          hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
+          // run-time weights (every b >= 1 here): the fp32 staircase screen
+          // first.  A corner it discards is dominated by a verified
+          // configuration p with T_p <= T and E > E_p (1 + 4u) (the val_p
+          // margin, section 5), so every configuration c of the tile has
+          // F_w(c) < F_w(p) strictly, in fp64 too, for every weight with
+          // b >= 1: the tile holds no optimum and no tie of one, and the
+          // weight screen (log-domain pre-screen + exact test) is skipped.
+          fdom = p.want_pareto && stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+          if (!fdom) hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
         } else {
           float mq[WS::N];
           WS::q(mT, mE, mq);
@@ -700,20 +748,14 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
           }
         }
-        cE = e_total(p, cT, cE);
-      }
-      hitm &= ~b0skip;
-      double c64 = -1.0;  // the tile's exact min fp64 makespan, computed on demand
-      if ((p.b0mode & 2) && hitm && b0_any<WS>(p, hitm)) {  // b = 0 weights: no configuration of the tile beats the lane's best
-        c64 = tile_corner64(wp, vt);
-        hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+        cE = fmaf(p.kidle0, cT, cE);
       }
       const bool hit = hitm != 0;
       bool par = false;
-      if (p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE))
-        par = !stair_dominated(stair, p, c64 >= 0.0 ? c64 : tile_corner64(wp, vt), cE);
+      if (p.want_pareto && !(WS::RT ? fdom : stair_dominated_fs(ss, p, __fmul_rd(cT, p.tlb_scale_f), cE)))
+        par = !stair_dominated(stair, p, tile_corner64(wp, t << 6), cE);
       if (hit || par) {
-        nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+        nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, t << 6, Tp, Ep, hit);
         thr_from_sm<WS>(p, thr, thr_sm);
       }
     }
@@ -721,19 +763,22 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     // Every rare path of the tile loop (unit-boundary tiles, exact corners,
     // slow re-checks) is entered warp-uniformly (a vote), so the common
     // iteration carries no convergence-barrier bookkeeping; lanes without work
-    // in a rare path skip it inside.
-    for (uint32_t st = s_lo; st <= s_hi; st++) {
-      const uint32_t j = 2 * st + h;
-      const uint32_t vt = (j << 10) | ((uint32_t)l4 << 6);
-      const bool live = j < (uint32_t)nloop && vt + 64 > v0 && vt < v1;
-      const bool part = live && (vt < v0 || vt + 64 > v1);
-      if (__any_sync(0xffffffffu, part)) {  // partial tiles at a unit boundary
-        if (part)
-          nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt > v0 ? vt : v0, vt + 64 < v1 ? vt + 64 : v1, 1);
-        thr_from_sm<WS>(p, thr, thr_sm);
-      }
-      const bool full = live && !part;
-      const float2 lp = wp.lp[j < (uint32_t)nloop ? j : 0u];
+    // in a rare path skip it inside.  Tiles as in the plain loop (tile t of
+    // lane t mod 32); the steps run warp-uniformly over the full tiles.
+    const uint32_t tb0 = v0 >> 6, tb1 = (v1 - 1) >> 6;
+    const bool e0 = (v0 & 63u) && (tb0 & 31u) == (uint32_t)lane;
+    const bool e1 = (v1 & 63u) && (tb1 & 31u) == (uint32_t)lane && !(tb1 == tb0 && (v0 & 63u));
+    if (__any_sync(0xffffffffu, e0 || e1)) {  // partial tiles at a unit boundary
+      if (e0) nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, v0, min(v1, (tb0 + 1) << 6), 1);
+      if (e1) nref += edge_configs<WS>(tb, *p.gp, stair, wp, thr_sm, lb, max(v0, tb1 << 6), v1, 1);
+      thr_from_sm<WS>(p, thr, thr_sm);
+    }
+    const uint32_t te = v1 >> 6;
+    const uint32_t tf = (v0 + 63u) >> 6;
+    for (uint32_t st = tf >> 5; (st << 5) < te; st++) {
+      const uint32_t t = (st << 5) + (uint32_t)lane;
+      const bool full = t >= tf && t < te;
+      const float2 lp = wp.lp[full ? t >> 4 : 0u];
       const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
       unsigned hitm = 0;
       float cE, cT;
@@ -749,16 +794,16 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
           const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
   #pragma unroll
           for (int b = 0; b < 4; b++) {
-            const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
+            const float E2 = E1 + Be[b];
   #pragma unroll
             for (int c = 0; c < 4; c++) {
-              const float T = fmaxf(T2, Ct[c]), E = E2 + Ce[c];
+              const float T = fmax3f(T1, Bt[b], Ct[c]), E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
             }
           }
         }
-        mE = e_total(p, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D)
+        mE = fmaf(p.kidle0, mT, mE);  // the exact corner's E (COUNT_IDLE: kidle T + D; else + 0)
         if constexpr (WS::RT) {
           hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
         } else {
@@ -783,26 +828,26 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             for (int c = 0; c < 4; c++) cE = fminf(cE, E2 + Ce[c]);
           }
         }
-        cE = e_total(p, cT, cE);
+        cE = fmaf(p.kidle0, cT, cE);
       }
       hitm = full ? (hitm & ~b0skip) : 0u;
       // exact tile corner (fp64 min makespan) where a screen needs it: b = 0
       // weights (no configuration of the tile beats the lane's best) and the
       // Pareto screen when the fp32 staircase test cannot decide
       const bool b0c = (p.b0mode & 2) && hitm && b0_any<WS>(p, hitm);
-      const bool fpar = full && p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(cT, p.tlb_scale_f), cE);
+      const bool fpar = full && p.want_pareto && !stair_dominated_fs(ss, p, __fmul_rd(cT, p.tlb_scale_f), cE);
       bool par = false;
       if (__any_sync(0xffffffffu, b0c || fpar)) {
         if (b0c || fpar) {
-          const double c64 = tile_corner64(wp, vt);
-          if (b0c) hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + vt);
+          const double c64 = tile_corner64(wp, t << 6);
+          if (b0c) hitm &= ~b0_beaten<WS>(p, lb, hitm, c64, wp.base + (t << 6));
           if (fpar) par = !stair_dominated(stair, p, c64, cE);
         }
       }
       const bool hit = hitm != 0;
       const bool slow = hit || par;
       if (__any_sync(0xffffffffu, slow)) {
-        if (slow) nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, vt, Tp, Ep, hit);
+        if (slow) nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, t << 6, Tp, Ep, hit);
         thr_from_sm<WS>(p, thr, thr_sm);
       }
     }
@@ -819,6 +864,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
   Stair stair = stair_at(after);
+  const StairSm ss = stair_sm(stair);
   WarpPart *wps = (WarpPart *)(after + kStairSmem);
   WarpPart &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kTileWarps);
@@ -905,7 +951,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
         if (feas) wp.nfeas += v1 - v0;
       }
       __syncwarp();
-      if (feas) nref += partition_configs<L, WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
+      if (feas) nref += partition_configs<L, WS>(tb, p, stair, ss, wp, thr, thr_sm, lb, v0, v1, lane);
       __syncwarp();
       if (base + Pn >= e) break;
       if (lane == 0) {
