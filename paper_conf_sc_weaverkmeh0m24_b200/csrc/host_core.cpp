@@ -546,7 +546,9 @@ int build_stage(const Profile &P, const Query &q, const Space &sp, std::vector<u
   dp->kidle0 = (q.model & SCHED_MODEL_COUNT_IDLE) ? dp->kidle : 0.f;
   dp->mem_cap = P.mem_cap;
   dp->want_pareto = q.want_pareto;
+  dp->wb_pos = 1;
   for (int w = 0; w < q.nw; w++) {
+    dp->wb_pos &= q.wb[w] >= 1 ? 1 : 0;
     dp->wa[w] = q.wa[w];
     dp->wb[w] = q.wb[w];
   }

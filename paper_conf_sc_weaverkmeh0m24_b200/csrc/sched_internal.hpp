@@ -87,6 +87,7 @@ struct DevParams {
   float kidle0;             // kidle under COUNT_IDLE, else 0 (tile loop: E + kidle0 T as one FFMA)
   double gps;               // g * P_s (exact) for COUNT_IDLE
   int mem_cap, want_pareto, root, nstates;
+  int wb_pos;               // every weight has b >= 1 (corner screens: staircase domination implies no weight hit)
   uint32_t bucket_base;     // (bits64(T_lower) >> bucket_shift)
   int bucket_shift;         // kBucketShift, or finer after the seed pass (re-bucketing, search.cu)
   // the same buckets from the bits of a float T (stair_dominated_f):

@@ -258,6 +258,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   unsigned char *after = sm + ((p.blob_bytes + 15) & ~15u);
   Stair stair = stair_at(after);
+  const StairSm ss = stair_sm(stair);
   C2Warp *wps = (C2Warp *)(after + kStairSmem);
   C2Warp &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kC2Warps);
@@ -399,25 +400,33 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
                 const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
 #pragma unroll
                 for (int b = 0; b < 4; b++) {
-                  const float T2 = fmaxf(T1, Bt[b]), E2 = E1 + Be[b];
+                  const float E2 = E1 + Be[b];
 #pragma unroll
                   for (int c = 0; c < 4; c++) {
-                    mT = fminf(mT, fmaxf(T2, Ct[c]));
+                    mT = fminf(mT, fmax3f(T1, Bt[b], Ct[c]));  // T: one FMNMX3 per configuration
                     mE = fminf(mE, E2 + Ce[c]);
                   }
                 }
               }
+              // the fp32 staircase screen first: a corner it discards is
+              // dominated by a verified configuration with margin (E > E_p
+              // (1 + 4u)), so when every weight has b >= 1
+              // no configuration of the tile reaches or ties any weight's
+              // optimum and the weight screen is skipped
+              const bool fdom = p.want_pareto && stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE);
               bool hit = false;
+              if (!(fdom && p.wb_pos)) {
 #pragma unroll
-              for (int w = 0; w < WM; w++) {
-                if (w < p.nw) {
-                  float q = 1.f;
-                  for (int i = 0; i < p.wa[w]; i++) q *= mT;
-                  for (int i = 0; i < p.wb[w]; i++) q *= mE;
-                  hit |= q <= thr[w] * p.mul[w];
+                for (int w = 0; w < WM; w++) {
+                  if (w < p.nw) {
+                    float q = 1.f;
+                    for (int i = 0; i < p.wa[w]; i++) q *= mT;
+                    for (int i = 0; i < p.wb[w]; i++) q *= mE;
+                    hit |= q <= thr[w] * p.mul[w];
+                  }
                 }
               }
-              bool par = p.want_pareto && !stair_dominated_f(stair, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+              bool par = p.want_pareto && !fdom;
               if (par) {  // the fp32 screen cannot decide: the tile's exact fp64 corner makespan
                 double c = 0.0;
 #pragma unroll
