@@ -602,7 +602,7 @@ __device__ __forceinline__ int small_l_configs(const Tables &tb, const DevParams
 template <int L, class WS>
 __device__ __forceinline__ int partition_configs(const Tables &tb, const DevParams &p, const Stair &stair,
                                                  const StairSm &ss, WarpPart &wp, Thr<WS> &thr, float *thr_sm,
-                                                 BestRec *lb, uint32_t v0, uint32_t v1, int lane, float4 *sa) {
+                                                 BestRec *lb, uint32_t v0, uint32_t v1, int lane) {
   if constexpr (L != 4) return small_l_configs<L, WS>(tb, p, stair, wp, thr, thr_sm, lb, v0, v1, lane);
   const int k = wp.cfg.k;
   if (k < 5) {
@@ -677,23 +677,9 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     if (edge) thr_from_sm<WS>(p, thr, thr_sm);
     const uint32_t te = v1 >> 6;
     const uint32_t tf = (v0 + 63u) >> 6;
-#ifdef SCHED_TILE_SA
-    // the lane's digits folded into group k-3's records, kept in the lane's
-    // shared-memory slots (not registers): T1 = max(lp.x, max(Tl, At[a])),
-    // E1 = lp.y + (El + Ae[a])
-    sa[0] = make_float4(fmaxf(Tl, At[0]), fmaxf(Tl, At[1]), fmaxf(Tl, At[2]), fmaxf(Tl, At[3]));
-    sa[kTileThreads] = make_float4(El + Ae[0], El + Ae[1], El + Ae[2], El + Ae[3]);
-#endif
-#ifdef SCHED_TILE_U2
-#pragma unroll 2
-#endif
     for (uint32_t t = tf + (((uint32_t)lane - tf) & 31u); t < te; t += 32) {
       const float2 lp = wp.lp[t >> 4];
       const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
-#ifdef SCHED_TILE_SA
-      const float4 ta4 = sa[0], ea4 = sa[kTileThreads];
-      const float TA[4] = {ta4.x, ta4.y, ta4.z, ta4.w}, EA[4] = {ea4.x, ea4.y, ea4.z, ea4.w};
-#endif
       unsigned hitm = 0;
       float cE, cT;
       bool fdom = false;  // WS::RT: corner discarded by the fp32 staircase screen
@@ -706,24 +692,13 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         float mT = __int_as_float(0x7f800000), mE = mT;
   #pragma unroll
         for (int a = 0; a < 4; a++) {
-#ifdef SCHED_TILE_SA
-          const float T1 = fmaxf(lp.x, TA[a]), E1 = lp.y + EA[a];
-#else
           const float T1 = fmaxf(Tp, At[a]), E1 = Ep + Ae[a];
-#endif
   #pragma unroll
           for (int b = 0; b < 4; b++) {
-#ifdef SCHED_TILE_T2
-            const float T2 = fmaxf(T1, Bt[b]);
-#endif
             const float E2 = E1 + Be[b];
   #pragma unroll
             for (int c = 0; c < 4; c++) {
-#ifdef SCHED_TILE_T2
-              const float T = fmaxf(T2, Ct[c]);
-#else
-              const float T = fmax3f(T1, Bt[b], Ct[c]);  // one ALU slot per configuration, no per-pair T2
-#endif
+              const float T = fmax3f(T1, Bt[b], Ct[c]);  // one ALU slot per configuration
               const float E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);
@@ -887,9 +862,6 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
   WarpPart &wp = wps[warp];
   BestRec *red = (BestRec *)(wps + kTileWarps);
   float *thr_sm = (float *)(red + kTileWarps * kMaxW) + threadIdx.x * (kMaxW + 1);  // odd row stride: no bank conflicts
-  // per-thread float4 slots after the threshold rows (SCHED_TILE_SA): [0, T) and [T, 2T)
-  float4 *sa = (float4 *)(((uintptr_t)((float *)(red + kTileWarps * kMaxW) + kTileThreads * (kMaxW + 1)) + 15) &
-                          ~(uintptr_t)15) + threadIdx.x;
   const GroupRec *gtab = (const GroupRec *)p.gtab;
   stair_init(stair);
   __syncthreads();
@@ -972,7 +944,7 @@ __global__ void __launch_bounds__(kTileThreads, kTileMinBlocks) k_tile(const Dev
         if (feas) wp.nfeas += v1 - v0;
       }
       __syncwarp();
-      if (feas) nref += partition_configs<L, WS>(tb, p, stair, ss, wp, thr, thr_sm, lb, v0, v1, lane, sa);
+      if (feas) nref += partition_configs<L, WS>(tb, p, stair, ss, wp, thr, thr_sm, lb, v0, v1, lane);
       __syncwarp();
       if (base + Pn >= e) break;
       if (lane == 0) {

@@ -71,11 +71,7 @@ static const void *tile_pick_ws(DevParams *dp) {
 
 size_t tile_smem_bytes(const DevParams &dp) {
   return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + sizeof(WarpPart) * kTileWarps +
-         sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * (kMaxW + 1)
-#ifdef SCHED_TILE_SA
-         + 16 + 2 * sizeof(float4) * kTileThreads
-#endif
-      ;
+         sizeof(BestRec) * kTileWarps * kMaxW + sizeof(float) * kTileThreads * (kMaxW + 1);
 }
 
 bool tile_eligible(DevParams &dp, TileLaunch *tl) {
