@@ -342,6 +342,180 @@ __device__ __forceinline__ void sfx_fast(const DevParams &p, const Stair &stair,
   }
 }
 
+// ---- fast pass over grandparents (SCHED_SFX_PAIRS, default) ----
+// A grandparent is a state after x_0..x_{M-3}; its configurations are the
+// placements (j1, j2) of the last two elements x_{M-2}, x_{M-1}.  sfx_pairs
+// evaluates them as an 8 x 8 register tile without branches: per slot j the
+// table entries of the row with the suffix subset S_j plus x_{M-2} (A), plus
+// both (D: j1 == j2, the same group), plus x_{M-1} alone (B); rows above the
+// grandparent's kc (unused empty rows) read +inf, full groups read +inf from
+// the table itself; the one placement the tile does not cover -- x_{M-2} in
+// the new group kc and x_{M-1} in a second new group kc + 1 -- is evaluated
+// on its own.  Per configuration T = max(T_g, t_A, t_B), E = (E_g + e_A) + e_B
+// (the chain order of sfx_apply), min-reduced; the feasible count comes from
+// the finite masks of A, B, D (no per-configuration count).
+template <int M>
+__device__ __forceinline__ void sfx_pairs(const float2 *tab, const SfxLane &g, int G, float &mT, float &mE, int &nf) {
+  constexpr int RS = SfxWarp<M>::RS;
+  constexpr uint32_t bA = 1u << (M - 2), bB = 1u << (M - 1);
+  const float inf = __int_as_float(0x7f800000);
+  const uint32_t lo = (uint32_t)g.gi, hi = (uint32_t)(g.gi >> 32);
+  float tA[kSfxMaxG], eA[kSfxMaxG], tD[kSfxMaxG], eD[kSfxMaxG], tB[kSfxMaxG], eB[kSfxMaxG];
+  uint32_t fA = 0, fB = 0, fD = 0;
+#pragma unroll
+  for (int j = 0; j < kSfxMaxG; j++) {
+    const uint32_t S = __byte_perm(j < 4 ? lo : hi, 0u, 0x4440u | (uint32_t)(j & 3));
+    const bool used = j <= g.kc;  // existing groups and the new group kc
+    const float2 a = tab[j * RS + (S | bA)], d = tab[j * RS + (S | bA | bB)], b = tab[j * RS + (S | bB)];
+    tA[j] = used ? a.x : inf;
+    eA[j] = used ? a.y : inf;
+    tD[j] = used ? d.x : inf;
+    eD[j] = used ? d.y : inf;
+    tB[j] = used ? b.x : inf;
+    eB[j] = used ? b.y : inf;
+    fA |= (tA[j] < inf ? 1u : 0u) << j;
+    fB |= (tB[j] < inf ? 1u : 0u) << j;
+    fD |= (tD[j] < inf ? 1u : 0u) << j;
+  }
+  float lT = mT, lE = mE;
+#pragma unroll
+  for (int j1 = 0; j1 < kSfxMaxG; j1++) {
+    const float T1 = fmaxf(g.T, tA[j1]), E1 = g.E + eA[j1];
+#pragma unroll
+    for (int j2 = 0; j2 < kSfxMaxG; j2++) {
+      const float T = fmaxf(T1, j2 == j1 ? tD[j1] : tB[j2]);
+      const float E = E1 + (j2 == j1 ? eD[j1] : eB[j2]);
+      lT = fminf(lT, T);
+      lE = fminf(lE, E);
+    }
+  }
+  // x_{M-2} in the new group kc, x_{M-1} in a second new group kc + 1
+  int ext = 0;
+  if (g.kc + 1 < G) {
+    const float2 a = tab[g.kc * RS + bA], b = tab[(g.kc + 1) * RS + bB];
+    const float T = fmaxf(fmaxf(g.T, a.x), b.x), E = (g.E + a.y) + b.y;
+    lT = fminf(lT, T);
+    lE = fminf(lE, E);
+    ext = T < inf ? 1 : 0;
+  }
+  mT = lT;
+  mE = lE;
+  if (g.T < inf) nf += __popc(fA) * __popc(fB) - __popc(fA & fB) + __popc(fA & fD) + ext;
+}
+
+// configurations under a grandparent: sum over the options j1 of x_{M-2} of
+// the option count of x_{M-1} (r existing groups with room, `one` of them
+// with room 1, the new group if kc < G)
+__device__ __forceinline__ int sfx_pairs_count(const SfxLane &g, int G, int C) {
+  const int r = __popc(g.rm);
+  const int na = g.kc < G ? 1 : 0;
+  // groups (< kc) whose room nibble is exactly 1
+  const uint32_t x = g.rr ^ 0x11111111u;                 // nibble == 1 -> 0
+  const uint32_t z = ~(((x & 0x77777777u) + 0x77777777u) | x) & 0x88888888u;  // high bit of each zero nibble
+  const uint32_t km = g.kc >= 8 ? 0xffffffffu : ((1u << (4 * g.kc)) - 1u);
+  const int one = __popc(z & km);
+  return r * (r + na) - one + na * (r + (C > 1 ? 1 : 0) + (g.kc + 1 < G ? 1 : 0));
+}
+
+// next option at level I (I <= M-3) and the first grandparent below it
+template <int M, int I>
+__device__ __forceinline__ bool sfx_gadv(const SfxCtx &x, SfxLane (&st)[M - 2], uint32_t (&rem)[M - 2],
+                                         SfxLane &gp) {
+  constexpr int RS = SfxWarp<M>::RS;
+  while (rem[I]) {
+    const int j = __ffs(rem[I]) - 1;
+    rem[I] &= rem[I] - 1;
+    const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
+    SfxLane s = st[I];
+    sfx_apply(s, j, 1u << I, v, x.C);
+    if constexpr (I == M - 3) {
+      gp = s;
+      return true;
+    } else {
+      st[I + 1] = s;
+      rem[I + 1] = sfx_opts(s, x.G);
+      if (sfx_gadv<M, I + 1>(x, st, rem, gp)) return true;
+    }
+  }
+  return false;
+}
+
+template <int M, int I>
+__device__ __forceinline__ bool sfx_gnext(const SfxCtx &x, SfxLane (&st)[M - 2], uint32_t (&rem)[M - 2],
+                                          SfxLane &gp) {
+  if (sfx_gadv<M, I>(x, st, rem, gp)) return true;
+  if constexpr (I == 0) {
+    return false;
+  } else {
+    return sfx_gnext<M, I - 1>(x, st, rem, gp);
+  }
+}
+
+// the parents of grandparent gp whose x_{M-2} option is in remA, parent by
+// parent (the first one's x_{M-1} options masked by ofirst); returns true
+// when the lane's range (cnt) ends inside
+template <int M>
+__device__ __forceinline__ bool sfx_gp_parents(const DevParams &p, const Stair &stair, const SfxCtx &x, SfxHot &h,
+                                               const SfxLane &gp, uint32_t remA, uint32_t ofirst, int &cnt) {
+  constexpr int RS = SfxWarp<M>::RS;
+  constexpr uint32_t bA = 1u << (M - 2);
+  while (remA) {
+    const int j = __ffs(remA) - 1;
+    remA &= remA - 1;
+    const float2 v = x.tab[j * RS + (((uint32_t)(gp.gi >> (8 * j)) & 0xffu) | bA)];
+    SfxLane par = gp;
+    sfx_apply(par, j, bA, v, x.C);
+    const uint32_t oall = sfx_opts(par, x.G);
+    const uint32_t o = oall & ofirst;
+    ofirst = 0xffffffffu;
+    const int n = __popc(o);
+    if (cnt <= n) {
+      sfx_last<M, false>(p, stair, x, h, nullptr, par, o & ~strip_low(o, cnt));
+      cnt = 0;
+      return true;
+    }
+    if (o == oall) sfx_slots<M>(x.tab, par, x.G, h.mT, h.mE, h.nf);
+    else sfx_last<M, false>(p, stair, x, h, nullptr, par, o);
+    cnt -= n;
+  }
+  return false;
+}
+
+// Fast pass over the lane range by grandparents: the first (partial) and the
+// last (partial) grandparent parent by parent, the whole ones in between as
+// pair tiles.
+template <int M>
+__device__ __forceinline__ void sfx_fast_pairs(const DevParams &p, const Stair &stair, const SfxCtx &x, SfxHot &h,
+                                               const SfxLane &s0, int cnt) {
+  constexpr int RS = SfxWarp<M>::RS;
+  SfxLane st[M - 2], gp;
+  uint32_t rem[M - 2];
+  st[0] = s0;
+#pragma unroll
+  for (int I = 0; I < M - 2; I++) {
+    const int j = x.start[I];
+    rem[I] = sfx_opts(st[I], x.G) & (~1u << j);  // options after the start choice
+    const float2 v = x.tab[j * RS + (((uint32_t)(st[I].gi >> (8 * j)) & 0xffu) | (1u << I))];
+    SfxLane s = st[I];
+    sfx_apply(s, j, 1u << I, v, x.C);
+    if (I < M - 3) st[I + 1] = s;
+    else gp = s;
+  }
+  if (sfx_gp_parents<M>(p, stair, x, h, gp, sfx_opts(gp, x.G) & (~0u << x.start[M - 2]), ~0u << x.start[M - 1],
+                        cnt))
+    return;
+  for (;;) {
+    if (!sfx_gnext<M, M - 3>(x, st, rem, gp)) return;
+    const int np = sfx_pairs_count(gp, x.G, x.C);
+    if (cnt <= np) {  // the lane's range ends in this grandparent
+      sfx_gp_parents<M>(p, stair, x, h, gp, sfx_opts(gp, x.G), 0xffffffffu, cnt);
+      return;
+    }
+    sfx_pairs<M>(x.tab, gp, x.G, h.mT, h.mE, h.nf);
+    cnt -= np;
+  }
+}
+
 // Slow pass over a lane range (out of line: keeps the fast pass's registers).
 template <int M>
 static __device__ __noinline__ void sfx_slow(const DevParams &p, const Stair &stair, const SfxCtx &x,
@@ -597,7 +771,11 @@ __global__ void __launch_bounds__(kSfxThreads, SCHED_SFX_MINB) k_sfx(const DevPa
           h.nf = 0;
           h.cnt = (int)(l1 - l0);
           h.ord = l0;
+#ifdef SCHED_SFX_PARENTS  // A/B: round 1's parent-by-parent fast pass
           sfx_fast<M>(p, stair, x, h, s0, (int)(l1 - l0));
+#else
+          sfx_fast_pairs<M>(p, stair, x, h, s0, (int)(l1 - l0));
+#endif
           nfeas += (u64)h.nf;
           if (h.nf) {
             bool hit = false;
