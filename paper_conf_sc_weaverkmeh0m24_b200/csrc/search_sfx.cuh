@@ -345,12 +345,11 @@ __device__ __forceinline__ void sfx_fast(const DevParams &p, const Stair &stair,
 // ---- fast pass over grandparents (SCHED_SFX_PAIRS, default) ----
 // A grandparent is a state after x_0..x_{M-3}; its configurations are the
 // placements (j1, j2) of the last two elements x_{M-2}, x_{M-1}.  sfx_pairs
-// evaluates them as an 8 x 8 register tile without branches: per slot j the
-// table entries of the row with the suffix subset S_j plus x_{M-2} (A), plus
-// both (D: j1 == j2, the same group), plus x_{M-1} alone (B); rows above the
-// grandparent's kc (unused empty rows) read +inf, full groups read +inf from
-// the table itself; the one placement the tile does not cover -- x_{M-2} in
-// the new group kc and x_{M-1} in a second new group kc + 1 -- is evaluated
+// evaluates them as a register tile: the 8 slots of x_{M-1} (B entries: the
+// row's suffix subset S_j plus x_{M-1}; rows above the grandparent's kc read
+// +inf, full groups read +inf from the table itself) for every option j1 of
+// x_{M-2} (A entry: S_j1 plus x_{M-2}), and both in the same group (D entry:
+// S_j1 plus both); the placement in two new groups (kc, kc + 1) is evaluated
 // on its own.  Per configuration T = max(T_g, t_A, t_B), E = (E_g + e_A) + e_B
 // (the chain order of sfx_apply), min-reduced; the feasible count comes from
 // the finite masks of A, B, D (no per-configuration count).
@@ -360,34 +359,41 @@ __device__ __forceinline__ void sfx_pairs(const float2 *tab, const SfxLane &g, i
   constexpr uint32_t bA = 1u << (M - 2), bB = 1u << (M - 1);
   const float inf = __int_as_float(0x7f800000);
   const uint32_t lo = (uint32_t)g.gi, hi = (uint32_t)(g.gi >> 32);
-  float tA[kSfxMaxG], eA[kSfxMaxG], tD[kSfxMaxG], eD[kSfxMaxG], tB[kSfxMaxG], eB[kSfxMaxG];
-  uint32_t fA = 0, fB = 0, fD = 0;
+  // B: x_{M-1} alone in slot j2 (rows above kc unused: +inf)
+  float tB[kSfxMaxG], eB[kSfxMaxG];
+  uint32_t fB = 0;
 #pragma unroll
   for (int j = 0; j < kSfxMaxG; j++) {
     const uint32_t S = __byte_perm(j < 4 ? lo : hi, 0u, 0x4440u | (uint32_t)(j & 3));
-    const bool used = j <= g.kc;  // existing groups and the new group kc
-    const float2 a = tab[j * RS + (S | bA)], d = tab[j * RS + (S | bA | bB)], b = tab[j * RS + (S | bB)];
-    tA[j] = used ? a.x : inf;
-    eA[j] = used ? a.y : inf;
-    tD[j] = used ? d.x : inf;
-    eD[j] = used ? d.y : inf;
+    const float2 b = tab[j * RS + (S | bB)];
+    const bool used = j <= g.kc;
     tB[j] = used ? b.x : inf;
     eB[j] = used ? b.y : inf;
-    fA |= (tA[j] < inf ? 1u : 0u) << j;
     fB |= (tB[j] < inf ? 1u : 0u) << j;
-    fD |= (tD[j] < inf ? 1u : 0u) << j;
   }
   float lT = mT, lE = mE;
-#pragma unroll
-  for (int j1 = 0; j1 < kSfxMaxG; j1++) {
-    const float T1 = fmaxf(g.T, tA[j1]), E1 = g.E + eA[j1];
+  uint32_t fA = 0, fD = 0;
+  // x_{M-2} over its options j1 (existing groups with room, the new group kc)
+  for (uint32_t oa = sfx_opts(g, G); oa;) {
+    const int j1 = __ffs(oa) - 1;
+    oa &= oa - 1;
+    const uint32_t S = (uint32_t)(g.gi >> (8 * j1)) & 0xffu;
+    const float2 a = tab[j1 * RS + (S | bA)], d = tab[j1 * RS + (S | bA | bB)];
+    fA |= (a.x < inf ? 1u : 0u) << j1;
+    fD |= (d.x < inf ? 1u : 0u) << j1;
+    const float T1 = fmaxf(g.T, a.x), E1 = g.E + a.y;
+    // the 8 slots of x_{M-1} with B entries, slot j1 included: that one is
+    // not a configuration (x_{M-1} in j1 without x_{M-2}), its (T, E) only
+    // lowers the min-reduced corner -- still a lower bound of every real
+    // configuration's -- so the screen stays complete; the real placement
+    // (both in j1) is the D entry
 #pragma unroll
     for (int j2 = 0; j2 < kSfxMaxG; j2++) {
-      const float T = fmaxf(T1, j2 == j1 ? tD[j1] : tB[j2]);
-      const float E = E1 + (j2 == j1 ? eD[j1] : eB[j2]);
-      lT = fminf(lT, T);
-      lE = fminf(lE, E);
+      lT = fminf(lT, fmaxf(T1, tB[j2]));
+      lE = fminf(lE, E1 + eB[j2]);
     }
+    lT = fminf(lT, fmaxf(T1, d.x));
+    lE = fminf(lE, E1 + d.y);
   }
   // x_{M-2} in the new group kc, x_{M-1} in a second new group kc + 1
   int ext = 0;
