@@ -38,10 +38,10 @@
 namespace sched {
 
 #ifndef SCHED_SFX_THREADS
-#define SCHED_SFX_THREADS 256
+#define SCHED_SFX_THREADS 512  // one 512-thread CTA per SM (c5: 485 ms vs 500 at 256 x 2; M = 7 tables need it)
 #endif
 #ifndef SCHED_SFX_MINB
-#define SCHED_SFX_MINB 2
+#define SCHED_SFX_MINB 1
 #endif
 constexpr int kSfxThreads = SCHED_SFX_THREADS;
 constexpr int kSfxWarps = kSfxThreads / 32;

@@ -1,22 +1,33 @@
 // sfx_host.cu -- eligibility and launch of the L = 1 suffix kernel
 // (search_sfx.cuh); instantiations in sfx_<M>.cu.
+#include <cstdlib>
+
 #include "search_sfx.cuh"
 
 namespace sched {
 
 static size_t sfx_smem(const DevParams &dp, int M) {
-  const size_t warp = M == 6 ? sizeof(SfxWarp<6>) : sizeof(SfxWarp<4>);
+  const size_t warp = M == 7 ? sizeof(SfxWarp<7>) : M == 6 ? sizeof(SfxWarp<6>) : sizeof(SfxWarp<4>);
   return ((dp.blob_bytes + 15) & ~15u) + kStairSmem + warp * kSfxWarps + sizeof(BestRec) * kSfxWarps * kMaxW;
 }
 
 bool sfx_eligible(DevParams &dp, TileLaunch *tl) {
   if (dp.L != 1 || dp.g > kSfxMaxG || (dp.capped && dp.c > 15) || !dp.gtab_ok) return false;
   if (dp.model & SCHED_MODEL_COUNT_IDLE) return false;  // E = sum_g E_g only
+  // suffix length: 7 for n >= 12 (2^7-entry rows, 16 warps x 8.3 KB of tables;
+  // c5 392 ms vs 485 with M = 6: 14x fewer prefixes, so fewer table rebuilds,
+  // unranks and partial grandparents), 6 for n >= 8, 4 for n = 6, 7
   int M;
-  if (dp.n >= 8) M = 6;
+  if (dp.n >= 12) M = 7;
+  else if (dp.n >= 8) M = 6;
   else if (dp.n >= 6) M = 4;
   else return false;
-  tl->fn = M == 6 ? sfx_fn<6>() : sfx_fn<4>();
+  // SCHED_SFX_M=6 / 7 (measurement): force the suffix length where it applies
+  if (const char *e = std::getenv("SCHED_SFX_M")) {
+    const int m = std::atoi(e);
+    if ((m == 6 && dp.n >= 8) || (m == 7 && dp.n >= 12)) M = m;
+  }
+  tl->fn = M == 7 ? sfx_fn<7>() : M == 6 ? sfx_fn<6>() : sfx_fn<4>();
   tl->smem = sfx_smem(dp, M);
   tl->slots_per_cta = kSfxWarps;
   return true;

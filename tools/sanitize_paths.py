@@ -26,6 +26,8 @@ CASES = [  # name, SCHED_KERNEL, expected path, n, g, c, levels, scope, weights,
     ("dfs", "dfs", 2, 10, 5, 3, (100,), PER_GPU, SWEEP, 4),
     ("ctile2", "ctile2", 6, 7, 4, 3, (25, 50, 75, 100), PER_CLIENT, W, 7),        # round 2: group-table PER_CLIENT
     ("tile_rt", "tile", 1, 9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 2), (3, 1), (1, 0)), 8),   # run-time weights
+    ("tile_rtn", "tile", 1, 9, 6, 3, (25, 50, 75, 100), PER_GPU, ((1, 1), (2, 1), (1, 2)), 9),  # run-time, b >= 1
+    ("sfx_c", "sfx", 3, 11, 6, 3, (100,), PER_GPU, ((1, 1), (2, 1)), 10),     # pair tiles, capped groups
 ]
 
 
