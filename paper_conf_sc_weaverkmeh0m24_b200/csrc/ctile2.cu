@@ -34,7 +34,10 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
   if (err != cudaSuccess) return err;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   *grid = std::min(kC2MaxGrid, nsm * occ);
+  dp.c2_seed_tiles = 0;
   if (fixed_units && dp.chunk_log2 >= 12) {
+    if (const char *e = std::getenv("SCHED_C2_SEED_TILES")) dp.c2_seed_tiles = std::atoi(e);
+    else dp.c2_seed_tiles = 1;
     // seed pass: units smaller than a partition fix only the top index
     // digits, and a tile whose client is a low-numbered workflow straddles
     // such a unit (configuration-by-configuration path); sample

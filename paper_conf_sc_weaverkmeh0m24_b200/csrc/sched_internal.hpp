@@ -87,6 +87,8 @@ struct DevParams {
   float kidle0;             // kidle under COUNT_IDLE, else 0 (tile loop: E + kidle0 T as one FFMA)
   double gps;               // g * P_s (exact) for COUNT_IDLE
   int mem_cap, want_pareto, root, nstates;
+  int c2_seed_tiles;        // k_ctile2 seed pass: whole tiles sampled around each unit's position
+  int abort_ovf;            // the fast kernels stop taking units once the candidate buffer overflowed
   int wb_pos;               // every weight has b >= 1 (corner screens: staircase domination implies no weight hit)
   uint32_t bucket_base;     // (bits64(T_lower) >> bucket_shift)
   int bucket_shift;         // kBucketShift, or finer after the seed pass (re-bucketing, search.cu)

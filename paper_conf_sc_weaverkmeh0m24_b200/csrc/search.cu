@@ -653,7 +653,8 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     launches++;
   }
   DevParams dp_full = dp;
-  const bool seed = dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
+  const char *noseed = std::getenv("SCHED_NO_SEED");  // measurement: no seed pass
+  const bool seed = !(noseed && noseed[0] == '1') && dp.want_pareto && dp.n_owned > 0 && dp.chunk_log2 >= 12 &&
                     (dp.n_owned << (dp.chunk_log2 - 12)) >= ((uint64_t)1 << 20);  // >= 2^32 configs
   // passes: 0 seed (large searches), 1 full search, 2 re-run after a
   // candidate-buffer overflow (unseeded: re-bucketed to the overflowing
@@ -670,7 +671,14 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     }
     passes++;
     int keep = pass == 0 ? 0 : (pass == 1 ? (seed ? 2 : 0) : 1);
-    const bool span_rerun = pass == 2 && !seed && dp.want_pareto;  // dense front flooded coarse buckets
+    // pass 2 (after an overflow): re-bucketed to the overflowing pass's
+    // candidate span with a fresh staircase -- a dense front flooded coarse
+    // buckets, or (seeded) the seed's front missed the region the flood came
+    // from and its fine buckets clamped it
+    const bool span_rerun = pass == 2 && dp.want_pareto;
+    // passes 1 and 2 stop early once they overflow (they are re-run); the
+    // seed pass and the last re-run go to the end
+    dp.abort_ovf = (pass == 1 || pass == 2) ? 1 : 0;
     const int ncand0 = (pass == 1 && seed && dp.want_pareto) || span_rerun
                            ? (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap) : 0;
     if (ncand0 > 0) {

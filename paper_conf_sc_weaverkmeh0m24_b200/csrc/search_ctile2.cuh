@@ -284,7 +284,8 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
 
   for (;;) {
     u64 unit = 0;
-    if (lane == 0) unit = atomicAdd(p.ctr + kCtrUnit, 1ull);
+    if (lane == 0)  // a pass that overflowed the candidate buffer stops early (it is re-run)
+      unit = (p.abort_ovf && __ldcg(p.ctr + kCtrOverflow)) ? ~0ull : atomicAdd(p.ctr + kCtrUnit, 1ull);
     unit = __shfl_sync(0xffffffffu, unit, 0);
     if (unit >= p.n_units) break;
     const u64 ue = unit * p.unit_stride;
@@ -349,6 +350,19 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
             }
             o_hi = lo;
           }
+          // seed pass (p.c2_seed_tiles): the unit's index range only picks a
+          // place in the partition; from there 32 whole steps of tiles are
+          // sampled (32 x 32 tiles = 2^16 configurations, as many as the
+          // unit) -- a 2^16-index range cuts every tile whose clients carry
+          // high index digits, which sent the seed pass configuration by
+          // configuration (56 of 213 ms of a c3-client slice)
+          uint32_t tv0 = v0, tv1 = v1;
+          if (p.c2_seed_tiles) {
+            o_lo &= ~31u;
+            o_hi = min(nout, o_lo + 32u * 32u);
+            tv0 = 0;
+            tv1 = Pn;
+          }
           const uint32_t st_lo = o_lo >> 5, st_hi = (o_hi + 31) >> 5;
           // warp-uniform part of the table indices at st_lo
           int idxS[kC2Slots];
@@ -370,8 +384,8 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
             }
             const uint32_t o = (st << 5) | (uint32_t)lane;
             const uint32_t vo = voS + voL;
-            if (o < o_lo || o >= o_hi || (vo | tbits) < v0 || vo >= v1) continue;
-            const bool whole = vo >= v0 && (vo | tbits) < v1;
+            if (o < o_lo || o >= o_hi || (vo | tbits) < tv0 || vo >= tv1) continue;
+            const bool whole = vo >= tv0 && (vo | tbits) < tv1;
             float Tp = 0.f, Ep = 0.f;
 #pragma unroll
             for (int q = 0; q < 5; q++) {
@@ -440,7 +454,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
               }
               if (!hit && !par) continue;
             }
-            nref += c2_tile_slow<WM>(tb, *p.gp, stair, wp, thr, lb, o, vo, v0, v1, Tp, Ep, At, Ae, Bt, Be, Ct, Ce);
+            nref += c2_tile_slow<WM>(tb, *p.gp, stair, wp, thr, lb, o, vo, tv0, tv1, Tp, Ep, At, Ae, Bt, Be, Ct, Ce);
           }
         }
       }

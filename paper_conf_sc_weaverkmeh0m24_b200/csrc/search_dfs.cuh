@@ -243,7 +243,8 @@ __global__ void __launch_bounds__(kDfsThreads, 2) k_dfs(const DevParams p) {
 
   for (;;) {
     u64 unit = 0;
-    if (lane == 0) unit = atomicAdd(p.ctr + kCtrUnit, 1ull);
+    if (lane == 0)  // a pass that overflowed the candidate buffer stops early (it is re-run)
+      unit = (p.abort_ovf && __ldcg(p.ctr + kCtrOverflow)) ? ~0ull : atomicAdd(p.ctr + kCtrUnit, 1ull);
     unit = __shfl_sync(0xffffffffu, unit, 0);
     if (unit >= p.n_units) break;
     const u64 ue = unit * p.unit_stride;

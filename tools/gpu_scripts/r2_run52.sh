@@ -7,6 +7,5 @@ timeout 2400 python -m pytest tests -m gpu -q > gpurun_out/r2az_gputests.log 2>&
 echo "rc=$?" >> gpurun_out/r2az_gputests.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/r2az_smoke.log 2>&1
 timeout 300 python tools/time_search.py c5 --reps 3 > gpurun_out/r2az_c5.jsonl 2>&1
-bash tools/gpu_scripts/sanitize.sh > gpurun_out/r2az_sanitize.txt 2>&1
 timeout 900 python bench.py --steps 10 --warmup 3 > gpurun_out/r2az_bench.json 2> gpurun_out/r2az_bench.err
 echo done
