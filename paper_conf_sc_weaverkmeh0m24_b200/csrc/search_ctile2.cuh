@@ -376,6 +376,27 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
               voS += (uint32_t)wp.wb[b][kC2Slots];
             }
           for (uint32_t st = st_lo; st < st_hi; st++) {
+            // seed pass: thresholds and staircase refreshed every 4 steps (the
+            // pass starts from nothing; every lane's first tiles are re-checked
+            // configuration by configuration until they are)
+            if (p.c2_seed_tiles && ((st - st_lo) & 3u) == 3u) {
+#pragma unroll
+              for (int w = 0; w < WM; w++) {
+                if (w < p.nw) {  // publish the warp's minimum, take the global one
+                  float m = thr[w];
+#pragma unroll
+                  for (int o = 16; o; o >>= 1) m = fminf(m, __shfl_xor_sync(0xffffffffu, m, o));
+                  if (lane == 0 && m < __uint_as_float(__ldcg(p.thr + w))) atomicMin(p.thr + w, __float_as_uint(m));
+                  thr[w] = fminf(thr[w], __uint_as_float(__ldcg(p.thr + w)));
+                }
+              }
+              if (p.want_pareto) {
+                u64 sv = wp.sver;
+                stair_sync(stair, p, sv, __ldcg(p.ctr + kCtrStairVer));
+                __syncwarp();
+                if (lane == 0) wp.sver = sv;
+              }
+            }
             if (st > st_lo) {  // st - 1 -> st: delta row of its trailing-ones count
               const int c = __ffs(~(st - 1)) - 1;
 #pragma unroll
