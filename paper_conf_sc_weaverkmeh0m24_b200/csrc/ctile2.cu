@@ -42,7 +42,7 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
     // digits, and a tile whose client is a low-numbered workflow straddles
     // such a unit (configuration-by-configuration path); sample
     // per_sm x nsm units of 2^ul configurations (SCHED_C2_SEED="ul,per_sm")
-    int sl = 16, per = 32;
+    int sl = 16, per = 64;  // c3-client slice: 161 ms (32 per SM: 162)
     if (const char *e = std::getenv("SCHED_C2_SEED")) std::sscanf(e, "%d,%d", &sl, &per);
     sl = std::max(10, std::min(sl, dp.chunk_log2));
     const uint64_t units = dp.n_owned << (dp.chunk_log2 - sl);
