@@ -364,6 +364,7 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
             tv1 = Pn;
           }
           const uint32_t st_lo = o_lo >> 5, st_hi = (o_hi + 31) >> 5;
+          const bool inner = tv0 == 0 && tv1 == Pn && o_lo == 0 && o_hi == nout && (nout & 31u) == 0;
           // warp-uniform part of the table indices at st_lo
           int idxS[kC2Slots];
           uint32_t voS = 0;
@@ -405,8 +406,13 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
             }
             const uint32_t o = (st << 5) | (uint32_t)lane;
             const uint32_t vo = voS + voL;
-            if (o < o_lo || o >= o_hi || (vo | tbits) < tv0 || vo >= tv1) continue;
-            const bool whole = vo >= tv0 && (vo | tbits) < tv1;
+            // a unit covering the whole partition (the main pass: units of a
+            // partition's 4^n configurations) needs no per-tile range checks
+            bool whole = true;
+            if (!inner) {
+              if (o < o_lo || o >= o_hi || (vo | tbits) < tv0 || vo >= tv1) continue;
+              whole = vo >= tv0 && (vo | tbits) < tv1;
+            }
             float Tp = 0.f, Ep = 0.f;
 #pragma unroll
             for (int q = 0; q < 5; q++) {
