@@ -36,12 +36,13 @@ cudaError_t launch_ctile2(DevParams &dp, const TileLaunch &tl, int nsm, cudaStre
   *grid = std::min(kC2MaxGrid, nsm * occ);
   dp.c2_seed_tiles = 0;
   if (fixed_units && dp.chunk_log2 >= 12) {
+    // seed pass: per_sm x nsm units of 2^ul indices spread over the shard
+    // (SCHED_C2_SEED="ul,per_sm"); a unit only picks a place in its
+    // partition, from which the kernel samples 32 whole steps of tiles
+    // (c2_seed_tiles; SCHED_C2_SEED_TILES=0 for the index ranges themselves,
+    // which cut every tile whose clients carry high index digits)
     if (const char *e = std::getenv("SCHED_C2_SEED_TILES")) dp.c2_seed_tiles = std::atoi(e);
     else dp.c2_seed_tiles = 1;
-    // seed pass: units smaller than a partition fix only the top index
-    // digits, and a tile whose client is a low-numbered workflow straddles
-    // such a unit (configuration-by-configuration path); sample
-    // per_sm x nsm units of 2^ul configurations (SCHED_C2_SEED="ul,per_sm")
     int sl = 16, per = 64;  // c3-client slice: 161 ms (32 per SM: 162)
     if (const char *e = std::getenv("SCHED_C2_SEED")) std::sscanf(e, "%d,%d", &sl, &per);
     sl = std::max(10, std::min(sl, dp.chunk_log2));
