@@ -14,7 +14,8 @@ against each step's slice (coverage).
 
 Multi-GPU: `--gpus N` (N > 1) started without torchrun re-launches itself
 under `torch.distributed.run --nproc-per-node N` (one rank per GPU, NCCL);
-started under torchrun, WORLD_SIZE must equal N.  `--dry-run` runs the same
+started under torchrun, WORLD_SIZE must equal N, and the process group (and
+the NCCL exchange) is used even at one rank.  `--dry-run` runs the same
 rank / exchange / coverage plumbing on CPU (gloo) with a stub in place of the
 kernels (no scoring) -- the CPU test of the launcher.
 
