@@ -677,13 +677,6 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     if (edge) thr_from_sm<WS>(p, thr, thr_sm);
     const uint32_t te = v1 >> 6;
     const uint32_t tf = (v0 + 63u) >> 6;
-#ifdef SCHED_TILE_AB
-    float ABt[16];  // max(A_t[a], B_t[b]): T = max3(T_p, AB, C_c), no per-a T1
-  #pragma unroll
-    for (int a = 0; a < 4; a++)
-  #pragma unroll
-      for (int b = 0; b < 4; b++) ABt[a * 4 + b] = fmaxf(At[a], Bt[b]);
-#endif
     for (uint32_t t = tf + (((uint32_t)lane - tf) & 31u); t < te; t += 32) {
       const float2 lp = wp.lp[t >> 4];
       const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
@@ -705,11 +698,7 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
             const float E2 = E1 + Be[b];
   #pragma unroll
             for (int c = 0; c < 4; c++) {
-#ifdef SCHED_TILE_AB
-              const float T = fmax3f(Tp, ABt[a * 4 + b], Ct[c]);
-#else
               const float T = fmax3f(T1, Bt[b], Ct[c]);  // one ALU slot per configuration
-#endif
               const float E = E2 + Ce[c];
               mT = fminf(mT, T);
               mE = fminf(mE, E);

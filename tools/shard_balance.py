@@ -6,7 +6,7 @@ per-rank device search times and the strong-scaling efficiency the split
 allows, T(1) / (R * max_r T_r) -- the ceiling of the driver's 1 -> R GPU
 scaling (the NCCL exchange of a few KB per step is not included; the box
 has one GPU, so it cannot be measured here).
-  python tools/shard_balance.py > profiles/r01_shard_balance.md"""
+  python tools/shard_balance.py > profiles/r02_shard_balance.md"""
 import os
 import sys
 
@@ -15,7 +15,7 @@ sys.path.insert(0, ROOT)
 import paper_conf_sc_weaverkmeh0m24_b200 as S  # noqa: E402
 from synth import config  # noqa: E402
 
-SLICES, CHUNK_LOG2 = 64, 22
+SLICES, CHUNK_LOG2 = 64, 24   # as bench.py
 prof, q = config("c4")
 sch = S.Scheduler(prof)
 ws = sch.workspace(q)
