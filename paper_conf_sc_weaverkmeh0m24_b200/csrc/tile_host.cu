@@ -101,8 +101,10 @@ cudaError_t launch_tile(DevParams &dp, const TileLaunch &tl, int nsm, cudaStream
   if (!fixed_units) {
     const uint64_t range = dp.n_owned << dp.chunk_log2;
     const uint64_t warps = (uint64_t)(*grid) * kTileWarps;
+    uint64_t upw = 16;  // SCHED_TILE_UPW (measurement): target units per warp
+    if (const char *e = std::getenv("SCHED_TILE_UPW")) upw = std::max(1, std::atoi(e));
     int ul = 12;
-    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * 16) ul++;
+    while (ul < dp.chunk_log2 && (range >> (ul + 1)) >= warps * upw) ul++;
     dp.unit_log2 = ul;
     dp.n_units = dp.n_owned << (dp.chunk_log2 - ul);
     dp.unit_stride = 1;
