@@ -166,6 +166,9 @@ typedef struct {
   int32_t passes;               /* search passes (2 = re-run after candidate overflow) */
   uint64_t h2d_bytes;           /* host->device bytes this call copied (staged tables) */
   uint64_t d2h_bytes;           /* device->host bytes this call copied (counters, picks) */
+  float main_ms;                /* device time of the final full search pass's kernel launch alone
+                                   (CUDA events; search_ms also holds the seed pass, group table,
+                                   re-runs); sched_front_dp: its kernels */
 } sched_stats;
 
 /* One point of the exact front computed by sched_front_dp, with one witness

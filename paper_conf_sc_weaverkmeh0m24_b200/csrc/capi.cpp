@@ -260,7 +260,7 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
     if (st) return st;
     h2d = blob.size();
   }
-  LaunchInfo info;
+  LaunchInfo info{};
   std::vector<BestRec> bres;
   std::vector<CandRec> front;
   uint64_t ctr[kCtrN];
@@ -304,6 +304,7 @@ int sched_search(sched_handle *h, const sched_query *qin, void *ws, size_t ws_by
     stats->t_seq_s = dp.tseq;
     stats->e_seq_j = dp.eseq;
     stats->search_ms = info.search_ms;
+    stats->main_ms = info.main_ms;
     stats->total_ms = total_ms;
     stats->kernel_path = info.path;
     stats->grid_ctas = info.grid;
@@ -430,7 +431,7 @@ int sched_debug_scores32(sched_handle *h, const sched_query *qin, void *ws, size
   dp.dump = (unsigned char *)d_scores;
   dp.dump_lo = q.lo;
   dp.dump_n = q.hi - q.lo;
-  LaunchInfo info;
+  LaunchInfo info{};
   std::vector<BestRec> bres;
   std::vector<CandRec> front;
   uint64_t ctr[kCtrN];
@@ -535,6 +536,7 @@ int sched_front_dp(sched_handle *h, const sched_query *qin, void *ws, size_t ws_
     stats->t_seq_s = ts;
     stats->e_seq_j = es;
     stats->search_ms = ms;
+    stats->main_ms = ms;
     stats->total_ms = ms;
     stats->kernel_path = 4;
     stats->kernel_launches = launches;
@@ -708,6 +710,7 @@ int sched_search_splits(sched_handle *h, const sched_query *qin, const int32_t *
     agg.n_refined += s1.n_refined;
     agg.n_candidates += s1.n_candidates;
     agg.search_ms += s1.search_ms;
+    agg.main_ms += s1.main_ms;
     agg.total_ms += s1.total_ms;
     agg.kernel_launches += s1.kernel_launches;
     agg.passes += s1.passes;

@@ -216,6 +216,7 @@ int dp_front_run(const Profile &P, const Query &q, DevParams p, const std::vecto
 struct LaunchInfo {
   int path, grid, launches, passes;
   float search_ms;
+  float main_ms;   // the final full pass's search kernel launch
   uint64_t d2h_bytes;
 };
 size_t workspace_bytes(const DevParams &dp, int max_grid);

@@ -759,6 +759,7 @@ int launch_search(DevParams dp, void *d_ws, size_t ws_bytes, void *stream, Launc
     float ms = 0.f;
     CK(cudaEventElapsedTime(&ms, e1, e2));
     search_ms += ms;
+    info->main_ms = ms;  // the last pass run is the full pass the result comes from
     if (pass >= 1 && !ctr[kCtrOverflow]) break;
   }
   int ncand = (int)std::min<uint64_t>(ctr[kCtrCand], dp.cand_cap);

@@ -76,7 +76,7 @@ class Stats(C.Structure):
                 ("n_candidates", C.c_uint64), ("t_seq_s", C.c_double), ("e_seq_j", C.c_double),
                 ("search_ms", C.c_float), ("total_ms", C.c_float), ("kernel_path", C.c_int32),
                 ("grid_ctas", C.c_int32), ("kernel_launches", C.c_int32), ("passes", C.c_int32),
-                ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64)]
+                ("h2d_bytes", C.c_uint64), ("d2h_bytes", C.c_uint64), ("main_ms", C.c_float)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
