@@ -215,6 +215,17 @@ __device__ __forceinline__ bool stair_dominated_fs(const StairSm &s, const DevPa
   return false;
 }
 
+// pm of the bucket of a float lower bound tlb (the staircase's prefix minimum
+// over strictly lower buckets): pm is non-increasing in the bucket, so every
+// T >= tlb has pm[bucket(T)] <= this value
+__device__ __forceinline__ unsigned int stair_pm_at(const StairSm &s, const DevParams &p, float tlb) {
+  const int b = (int)((__float_as_uint(tlb) >> p.bkt_sh32) + p.bkt_off32);
+  const uint32_t j = (uint32_t)(b < 0 ? 0 : (b >= kBuckets ? kBuckets - 1 : b));
+  unsigned int pm;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(pm) : "r"(s.pm + 4u * j));
+  return pm;
+}
+
 // bit s set: weight s has b = 0 (F = X^a depends on T alone) and the lane's
 // best for it has T <= T64 and a lower index than idx: configurations with
 // makespan >= T64 and index >= idx have F <= that best's F (rounding is
@@ -677,6 +688,19 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
     if (edge) thr_from_sm<WS>(p, thr, thr_sm);
     const uint32_t te = v1 >> 6;
     const uint32_t tf = (v0 + 63u) >> 6;
+#ifndef SCHED_TILE_NO_PMP
+    // a partition-wide staircase bound: every tile corner's T is at least
+    // the partition's fp32 min makespan (max over groups of the group's min
+    // over levels), so pm of that bucket bounds pm of every tile's bucket
+    // from above: E above it is dominated without the per-tile bucket lookup
+    unsigned int pmp = 0xffffffffu;
+    if (WS::N > 0 && p.want_pareto) {  // (Pareto-only sets measured slower with it: 350 -> 358 ms)
+      float tmin = 0.f;
+      for (int b = 0; b < k; b++)
+        tmin = fmaxf(tmin, fminf(fminf(wp.gt[b * 4], wp.gt[b * 4 + 1]), fminf(wp.gt[b * 4 + 2], wp.gt[b * 4 + 3])));
+      pmp = stair_pm_at(ss, p, __fmul_rd(tmin, p.tlb_scale_f));
+    }
+#endif
     for (uint32_t t = tf + (((uint32_t)lane - tf) & 31u); t < te; t += 32) {
       const float2 lp = wp.lp[t >> 4];
       const float Tp = fmaxf(lp.x, Tl), Ep = lp.y + El;
@@ -717,7 +741,12 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
           // F_w(c) < F_w(p) strictly, in fp64 too, for every weight with
           // b >= 1: the tile holds no optimum and no tie of one, and the
           // weight screen (log-domain pre-screen + exact test) is skipped.
+#ifndef SCHED_TILE_NO_PMP
+          fdom = p.want_pareto &&
+                 (__float_as_uint(mE) > pmp || stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE));
+#else
           fdom = p.want_pareto && stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+#endif
           if (!fdom) hitm = rt_screen<WS>(p, thr, thr_sm, mT, mE);
         } else {
           float mq[WS::N];
@@ -745,7 +774,12 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
       }
       const bool hit = hitm != 0;
       bool par = false;
+#ifndef SCHED_TILE_NO_PMP
+      if (p.want_pareto && !(WS::RT ? fdom : ((WS::N > 0 && __float_as_uint(cE) > pmp) ||
+                                              stair_dominated_fs(ss, p, __fmul_rd(cT, p.tlb_scale_f), cE))))
+#else
       if (p.want_pareto && !(WS::RT ? fdom : stair_dominated_fs(ss, p, __fmul_rd(cT, p.tlb_scale_f), cE)))
+#endif
         par = !stair_dominated(stair, p, tile_corner64(wp, t << 6), cE);
       if (hit || par) {
         nref += tile_slow<WS>(tb, *p.gp, stair, wp, thr_sm, lb, t << 6, Tp, Ep, hit);
