@@ -69,11 +69,17 @@ __device__ __forceinline__ void c2_offsets(const C2Warp &wp, int *off) {
 // vector in shared memory, and the exact canonical fp64 T_g (refine64 order)
 // in the warp's global table t64 (read only by the tile's exact-corner
 // Pareto check, through L2)
-__device__ __forceinline__ void c2_tables(const Tables &tb, const DevParams &p, C2Warp &wp, int lane,
-                                          double *t64) {
+// Returns the partition's fp32 min makespan: max over groups of the group's
+// min T-hat over its member-level vectors (every configuration's T-hat is at
+// least that: T-hat is a max of these entries).
+__device__ __forceinline__ float c2_tables(const Tables &tb, const DevParams &p, C2Warp &wp, int lane,
+                                           double *t64) {
   const int k = wp.cfg.k;
   int off[kMaxG + 1];
   c2_offsets(wp, off);
+  float gmin[kMaxG];
+#pragma unroll
+  for (int g = 0; g < kMaxG; g++) gmin[g] = __int_as_float(0x7f800000);
   for (int e = lane; e < off[k]; e += 32) {
     float2 v = make_float2(0.f, 0.f);
     double T64 = 0.0;
@@ -90,13 +96,25 @@ __device__ __forceinline__ void c2_tables(const Tables &tb, const DevParams &p, 
           double E64;
           ct_group64(tb, p, m, lw, T64, E64);
         }
+#pragma unroll
+        for (int q = 0; q < kMaxG; q++)
+          if (q == g) gmin[q] = fminf(gmin[q], v.x);
       }
     }
     wp.tab[e] = v;
     if (p.want_pareto) __stcg(t64 + e, T64);
   }
+  float tmin = 0.f;
+#pragma unroll
+  for (int g = 0; g < kMaxG; g++) {
+    float m = gmin[g];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) m = fminf(m, __shfl_xor_sync(0xffffffffu, m, o));
+    if (g < k) tmin = fmaxf(tmin, m);
+  }
   __threadfence_block();
   __syncwarp();
+  return tmin;
 }
 
 // per-partition tile setup (k >= 3): outer digit map, delta / contribution
@@ -324,7 +342,9 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
       if (feas) {
         int idxL[kC2Slots];
         uint32_t voL, tbits;
-        c2_tables(tb, p, wp, lane, t64);
+        const float ptmin = c2_tables(tb, p, wp, lane, t64);
+        // the partition-wide staircase bound (as in the tile kernel)
+        const unsigned int pmp = p.want_pareto ? stair_pm_at(ss, p, __fmul_rd(ptmin, p.tlb_scale_f)) : 0xffffffffu;
         if (k < 3) {
           nref += c2_small<WM>(tb, *p.gp, stair, wp, thr, lb, v0, v1, lane);
         } else {
@@ -454,7 +474,8 @@ __global__ void __launch_bounds__(kC2Threads, 1) k_ctile2(const DevParams p) {
               // (1 + 4u)), so when every weight has b >= 1
               // no configuration of the tile reaches or ties any weight's
               // optimum and the weight screen is skipped
-              const bool fdom = p.want_pareto && stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE);
+              const bool fdom = p.want_pareto && (__float_as_uint(mE) > pmp ||
+                                                  stair_dominated_fs(ss, p, __fmul_rd(mT, p.tlb_scale_f), mE));
               bool hit = false;
               if (!(fdom && p.wb_pos)) {
 #pragma unroll
