@@ -733,6 +733,15 @@ __device__ __forceinline__ int partition_configs(const Tables &tb, const DevPara
         // the exact corner's E: COUNT_IDLE adds kidle T as one FFMA; without
         // it kidle0 = 0 and fma(0, T, E) == E exactly (T finite: feasible partition)
         mE = fmaf(p.kidle0, mT, mE);
+#if !defined(SCHED_TILE_NO_PMP) && !defined(SCHED_TILE_NO_PMSKIP)
+        // every weight has b >= 1 here: a corner the partition-wide bound
+        // clears is dominated with margin by a verified configuration, so
+        // no configuration of the tile reaches or ties a weight's optimum
+        // (section 5) either -- the whole tile is done with one compare
+        if constexpr (!WS::RT) {
+          if (__float_as_uint(mE) > pmp) continue;
+        }
+#endif
         if constexpr (WS::RT) {
           // run-time weights (every b >= 1 here): the fp32 staircase screen
           // first.  A corner it discards is dominated by a verified
